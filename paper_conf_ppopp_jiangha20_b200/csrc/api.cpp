@@ -1,0 +1,589 @@
+// C ABI of libsr (include/sr.h): ingest, the reorder driver (Fig 5 workflow, P:137;
+// decision rules P:265), plan construction, metadata export, host entry points.
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <numeric>
+#include <string>
+#include <vector>
+
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+#include "internal.h"
+
+namespace sr {
+
+static thread_local std::string g_err;
+void set_error(const std::string& msg) { g_err = msg; }
+
+namespace {
+
+constexpr int32_t kSplitChunk = 256;  // phase-S work item: at most this many nnz
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+double now_s() {
+  return std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
+
+int einval(const std::string& m) {
+  set_error(m);
+  return SR_EINVAL;
+}
+
+// Items of phase S for a sequence of (position-ordered) rows.
+struct ItemBuilder {
+  std::vector<Item> items;
+  std::vector<uint32_t> meta;
+  std::vector<int2> split_info;  // per slot
+  int64_t n_slots = 0;
+  void add_row(int32_t e0, int32_t e1, int32_t xrow, int32_t out, bool rmw) {
+    const int32_t len = e1 - e0;
+    if (len <= kSplitChunk) {
+      items.push_back(Item{e0, e1, xrow, out});
+      meta.push_back(rmw ? kItemRMW : 0u);
+      return;
+    }
+    const int32_t nch = (len + kSplitChunk - 1) / kSplitChunk;
+    const int32_t first = (int32_t)n_slots;
+    for (int32_t c = 0; c < nch; ++c) {
+      const int32_t a = e0 + c * kSplitChunk, b = std::min(e1, a + kSplitChunk);
+      items.push_back(Item{a, b, xrow, out});
+      meta.push_back((rmw ? kItemRMW : 0u) | kItemSplit | (uint32_t)(first + c));
+      split_info.push_back(make_int2(first, nch));
+    }
+    n_slots += nch;
+  }
+};
+
+int upload_items(DevPlan& P, ItemBuilder& ib, int64_t n_sddmm_items, cudaStream_t s) {
+  P.n_items = (int64_t)ib.items.size();
+  P.n_sitems = n_sddmm_items;
+  SR_TRY(P.items.upload(ib.items, s));
+  SR_TRY(P.item_meta.upload(ib.meta, s));
+  P.n_slots = ib.n_slots;
+  if (ib.n_slots > 0) {
+    SR_TRY(P.split_info.upload(ib.split_info, s));
+    SR_TRY(P.split_counter.alloc((size_t)ib.n_slots));
+    SR_CUDA_TRY(cudaMemsetAsync(P.split_counter.p, 0, ib.n_slots * sizeof(int32_t), s));
+  }
+  P.scratch.release();
+  P.scratch_k = 0;
+  return SR_OK;
+}
+
+// Identity plan: plain row-wise kernels over the canonical CSR.
+int build_identity_plan(sr_csr_s* h, cudaStream_t s) {
+  const HostCSR& A = h->A;
+  DevPlan& P = h->plan;
+  const int64_t nnz = A.nnz();
+  std::vector<int2> ent((size_t)nnz);
+#pragma omp parallel for schedule(static)
+  for (int64_t e = 0; e < nnz; ++e) {
+    ent[e].x = A.col[e];
+    ent[e].y = *reinterpret_cast<const int32_t*>(&A.val[e]);
+  }
+  SR_TRY(P.s_ent.upload(ent, s));
+  if (A.identity_pos) {
+    std::vector<int32_t> o((size_t)nnz);
+    std::iota(o.begin(), o.end(), 0);
+    SR_TRY(P.s_oidx.upload(o, s));
+  } else {
+    SR_TRY(P.s_oidx.upload(A.opos, s));
+  }
+  ItemBuilder ib;
+  std::vector<int32_t> zero_rows;
+  for (int64_t r = 0; r < A.M; ++r) {
+    if (A.rowptr[r + 1] > A.rowptr[r])
+      ib.add_row((int32_t)A.rowptr[r], (int32_t)A.rowptr[r + 1], (int32_t)r, (int32_t)r, false);
+    else
+      zero_rows.push_back((int32_t)r);
+  }
+  const int64_t n_nonzero = (int64_t)ib.items.size();
+  for (int32_t r : zero_rows) {
+    ib.items.push_back(Item{0, 0, r, r});
+    ib.meta.push_back(0u);
+  }
+  SR_TRY(upload_items(P, ib, n_nonzero, s));
+  P.n_dpanels = 0;
+  SR_CUDA_TRY(cudaStreamSynchronize(s));
+  return SR_OK;
+}
+
+// Device plan of a (possibly sharded) tiling.
+int build_exec_plan(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s) {
+  const HostCSR& A = h->A;
+  const Tiling& T = h->tiles;
+  DevPlan& P = h->plan;
+  const int64_t M = A.M;
+  const int32_t PR = h->params.panel_rows;
+  const bool sharded = h->params.world > 1;
+  const int64_t q0s = std::min<int64_t>(M, pb * PR), q1s = std::min<int64_t>(M, pe * PR);
+  const std::vector<int32_t>& perm1 = h->perm1;
+  // shard rows / packed nnz order: by position, dense (slot order) then remainder (CSR order)
+  h->shard_rows.assign(perm1.begin() + q0s, perm1.begin() + q1s);
+  std::vector<int32_t> d_out((size_t)T.n_dense(), 0), r_out(T.r_col.size(), 0);
+  h->shard_nnz_ids.clear();
+  {
+    int64_t k = 0;
+    for (int64_t q = q0s; q < q1s; ++q) {
+      for (int64_t e = T.drow_ptr[q]; e < T.drow_ptr[q + 1]; ++e) {
+        const int64_t orig = A.identity_pos ? T.d_cidx[e] : A.opos[T.d_cidx[e]];
+        d_out[e] = (int32_t)(sharded ? k : orig);
+        h->shard_nnz_ids.push_back(orig);
+        ++k;
+      }
+      for (int64_t e = T.rrow_ptr[q]; e < T.rrow_ptr[q + 1]; ++e) {
+        const int64_t orig = A.identity_pos ? T.r_cidx[e] : A.opos[T.r_cidx[e]];
+        r_out[e] = (int32_t)(sharded ? k : orig);
+        h->shard_nnz_ids.push_back(orig);
+        ++k;
+      }
+    }
+  }
+  // phase D
+  std::vector<DPanel> dp;
+  int64_t maxd = 0;
+  for (int64_t p = pb; p < pe; ++p) {
+    const int64_t dc0 = T.dense_ptr[p], dc1 = T.dense_ptr[p + 1];
+    if (dc1 == dc0) continue;
+    const int64_t q0 = p * PR, nrows = std::min<int64_t>(M, q0 + PR) - q0;
+    dp.push_back(DPanel{(int32_t)q0, (int32_t)nrows, (int32_t)dc0, (int32_t)dc1});
+    maxd = std::max(maxd, dc1 - dc0);
+  }
+  P.n_dpanels = (int64_t)dp.size();
+  P.max_dense_per_panel = maxd;
+  P.tile_cols = h->params.tile_cols;
+  P.panel_rows = PR;
+  SR_TRY(P.dpanels.upload(dp, s));
+  SR_TRY(P.dense_cols.upload(T.dense_cols, s));
+  {
+    std::vector<int32_t> drp((size_t)M + 1);
+    for (int64_t q = 0; q <= M; ++q) drp[q] = (int32_t)T.drow_ptr[q];
+    SR_TRY(P.drow_ptr.upload(drp, s));
+    std::vector<int2> de((size_t)T.n_dense());
+#pragma omp parallel for schedule(static)
+    for (int64_t e = 0; e < T.n_dense(); ++e) {
+      de[e].x = T.d_slot[e];
+      de[e].y = *reinterpret_cast<const int32_t*>(&A.val[T.d_cidx[e]]);
+    }
+    SR_TRY(P.d_ent.upload(de, s));
+    SR_TRY(P.d_oidx.upload(d_out, s));
+    std::vector<int32_t> pout((size_t)M);
+    for (int64_t q = 0; q < M; ++q) pout[q] = sharded ? (int32_t)(q - q0s) : perm1[q];
+    SR_TRY(P.pos_xrow.upload(perm1, s));
+    SR_TRY(P.pos_out.upload(pout, s));
+  }
+  // phase S: remainder rows in perm2 order (restricted to the shard), then zero rows
+  std::vector<int2> se;
+  std::vector<int32_t> so;
+  se.reserve(T.r_col.size());
+  so.reserve(T.r_col.size());
+  ItemBuilder ib;
+  for (int32_t q : h->perm2) {
+    if (q < q0s || q >= q1s) continue;
+    const int32_t e0 = (int32_t)se.size();
+    for (int64_t e = T.rrow_ptr[q]; e < T.rrow_ptr[q + 1]; ++e) {
+      int2 v;
+      v.x = T.r_col[e];
+      v.y = *reinterpret_cast<const int32_t*>(&A.val[T.r_cidx[e]]);
+      se.push_back(v);
+      so.push_back(r_out[e]);
+    }
+    const bool rmw = T.drow_ptr[q + 1] > T.drow_ptr[q];
+    const int32_t out = sharded ? (int32_t)(q - q0s) : perm1[q];
+    ib.add_row(e0, (int32_t)se.size(), perm1[q], out, rmw);
+  }
+  const int64_t n_nonzero = (int64_t)ib.items.size();
+  for (int64_t q = q0s; q < q1s; ++q) {
+    if (T.drow_ptr[q + 1] == T.drow_ptr[q] && T.rrow_ptr[q + 1] == T.rrow_ptr[q]) {
+      const int32_t out = sharded ? (int32_t)(q - q0s) : perm1[q];
+      ib.items.push_back(Item{0, 0, perm1[q], out});
+      ib.meta.push_back(0u);
+    }
+  }
+  SR_TRY(P.s_ent.upload(se, s));
+  SR_TRY(P.s_oidx.upload(so, s));
+  SR_TRY(upload_items(P, ib, n_nonzero, s));
+  SR_CUDA_TRY(cudaStreamSynchronize(s));
+  return SR_OK;
+}
+
+int check_params(const sr_reorder_params* p) {
+  if (!p) return einval("sr_reorder: params is NULL");
+  if (p->siglen <= 0 || p->siglen > 256) return einval("siglen must be in 1..256");
+  if (p->bsize <= 0 || p->siglen % p->bsize != 0) return einval("siglen % bsize != 0 (R24)");
+  if (p->bsize > 2) {
+    set_error("bsize > 2 is not supported by the GPU banding kernel");
+    return SR_EUNSUPPORTED;
+  }
+  if (p->threshold_size < 2) return einval("threshold_size must be >= 2");
+  if (p->max_bucket < 0 || p->max_bucket == 1) return einval("max_bucket must be 0 or >= 2");
+  if (p->panel_rows < 1 || p->panel_rows > 128) return einval("panel_rows must be in 1..128");
+  if (p->dense_min < 1) return einval("dense_min must be >= 1");
+  if (p->tile_cols < 1 || p->tile_cols > 1024) return einval("tile_cols must be in 1..1024");
+  if (p->mode < 0 || p->mode > 2) return einval("mode must be AUTO, FORCE or OFF");
+  if (p->skip_dense_den <= 0 || p->skip_sim_den <= 0 || p->skip_dense_num < 0 || p->skip_sim_num < 0)
+    return einval("decision thresholds must be non-negative fractions");
+  if (p->world < 1 || p->rank < 0 || p->rank >= p->world) return einval("bad world / rank");
+  return SR_OK;
+}
+
+// LSH + Alg 3 over a column-sorted CSR (rows = the matrix being reordered).
+int reorder_round(const int64_t* rowptr, const int32_t* col, int64_t M, const sr_reorder_params& p,
+                  cudaStream_t s, std::vector<int32_t>& perm, int64_t* E, double* t_lsh, double* t_cl) {
+  std::vector<uint64_t> pairs;
+  std::vector<uint32_t> inter, uni;
+  const double t0 = now_s();
+  SR_TRY(lsh_candidates(rowptr, col, M, rowptr[M], p, s, pairs, inter, uni, E));
+  const double t1 = now_s();
+  perm.resize((size_t)M);
+  cluster_rows(M, rowptr, col, (int64_t)pairs.size(), pairs.data(), inter.data(), uni.data(),
+               p.threshold_size, perm.data());
+  *t_lsh += t1 - t0;
+  *t_cl += now_s() - t1;
+  return SR_OK;
+}
+
+}  // namespace
+}  // namespace sr
+
+using namespace sr;
+
+extern "C" {
+
+const char* sr_last_error(void) { return g_err.c_str(); }
+const char* sr_version(void) { return "sr 0.1 (sm_100a)"; }
+
+void sr_default_params(sr_reorder_params* p) {
+  if (!p) return;
+  std::memset(p, 0, sizeof(*p));
+  p->siglen = 128;
+  p->bsize = 2;
+  p->threshold_size = 256;
+  p->max_bucket = 32;
+  p->seed = 4;
+  p->panel_rows = 64;
+  p->dense_min = 2;
+  p->tile_cols = 64;
+  p->mode = SR_REORDER_AUTO;
+  p->skip_dense_num = 1;
+  p->skip_dense_den = 10;
+  p->skip_sim_num = 1;
+  p->skip_sim_den = 10;
+  p->world = 1;
+  p->rank = 0;
+}
+
+int sr_csr_create(int64_t nrows, int64_t ncols, int64_t nnz, const int64_t* rowptr,
+                  const int32_t* colidx, const float* vals, int device, sr_csr* out) {
+  if (!out) return einval("sr_csr_create: out is NULL");
+  *out = nullptr;
+  if (nrows < 0 || ncols < 0 || nnz < 0) return einval("negative size");
+  if (nrows >= (1ll << 31) || ncols >= (1ll << 31) || nnz >= (1ll << 31)) {
+    set_error("nrows, ncols and nnz must be < 2^31");
+    return SR_EUNSUPPORTED;
+  }
+  if (!rowptr || (nnz > 0 && (!colidx || !vals))) return einval("NULL CSR array");
+  if (rowptr[0] != 0 || rowptr[nrows] != nnz) return einval("rowptr[0] != 0 or rowptr[M] != nnz");
+  for (int64_t i = 0; i < nrows; ++i)
+    if (rowptr[i + 1] < rowptr[i]) return einval("rowptr is decreasing at row " + std::to_string(i));
+  auto* h = new (std::nothrow) sr_csr_s();
+  if (!h) {
+    set_error("out of host memory");
+    return SR_ENOMEM;
+  }
+  h->device = device;
+  HostCSR& A = h->A;
+  A.M = nrows;
+  A.N = ncols;
+  A.rowptr.assign(rowptr, rowptr + nrows + 1);
+  A.col.resize((size_t)nnz);
+  A.val.resize((size_t)nnz);
+  bool bad = false, unsorted = false;
+#pragma omp parallel for schedule(dynamic, 1024) reduction(|| : bad, unsorted)
+  for (int64_t i = 0; i < nrows; ++i) {
+    for (int64_t e = rowptr[i]; e < rowptr[i + 1]; ++e) {
+      if (colidx[e] < 0 || colidx[e] >= ncols) bad = true;
+      if (e > rowptr[i] && colidx[e] <= colidx[e - 1]) unsorted = true;
+    }
+  }
+  if (bad) {
+    delete h;
+    return einval("column index out of range");
+  }
+  if (!unsorted) {
+    std::memcpy(A.col.data(), colidx, nnz * sizeof(int32_t));
+    std::memcpy(A.val.data(), vals, nnz * sizeof(float));
+    A.identity_pos = true;
+  } else {
+    A.identity_pos = false;
+    A.opos.resize((size_t)nnz);
+    bool dup = false;
+#pragma omp parallel for schedule(dynamic, 1024) reduction(|| : dup)
+    for (int64_t i = 0; i < nrows; ++i) {
+      const int64_t b = rowptr[i], e = rowptr[i + 1];
+      std::vector<int64_t> idx((size_t)(e - b));
+      std::iota(idx.begin(), idx.end(), b);
+      std::sort(idx.begin(), idx.end(), [&](int64_t x, int64_t y) {
+        return colidx[x] != colidx[y] ? colidx[x] < colidx[y] : x < y;
+      });
+      for (int64_t t = 0; t < e - b; ++t) {
+        A.col[b + t] = colidx[idx[t]];
+        A.val[b + t] = vals[idx[t]];
+        A.opos[b + t] = (int32_t)idx[t];
+        if (t > 0 && A.col[b + t] == A.col[b + t - 1]) dup = true;
+      }
+    }
+    if (dup) {
+      delete h;
+      return einval("duplicate (row, col) entry");
+    }
+  }
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) {
+    cudaGetLastError();
+    delete h;
+    set_error("sr_csr_create: no such CUDA device " + std::to_string(device));
+    return SR_ECUDA;
+  }
+  DeviceGuard dg(device);
+  if (cudaStreamCreateWithFlags(&h->init_stream, cudaStreamNonBlocking) != cudaSuccess) {
+    cudaGetLastError();
+    delete h;
+    set_error("cudaStreamCreate failed");
+    return SR_ECUDA;
+  }
+  int rc = build_identity_plan(h, h->init_stream);
+  if (rc != SR_OK) {
+    sr_destroy(h);
+    return rc;
+  }
+  sr_default_params(&h->params);
+  h->perm1.resize((size_t)nrows);
+  std::iota(h->perm1.begin(), h->perm1.end(), 0);
+  h->stats.nnz = nnz;
+  *out = h;
+  return SR_OK;
+}
+
+int sr_reorder(sr_csr h, const sr_reorder_params* p, sr_stream stream) {
+  if (!h) return einval("sr_reorder: NULL handle");
+  SR_TRY(check_params(p));
+  if (h->reordered) {
+    set_error("sr_reorder: the handle already has a plan");
+    return SR_ESTATE;
+  }
+  DeviceGuard dg(h->device);
+  cudaStream_t s = stream ? (cudaStream_t)stream : h->init_stream;
+  const double t_start = now_s();
+  h->params = *p;
+  const HostCSR& A = h->A;
+  const int64_t M = A.M, nnz = A.nnz();
+  sr_plan_stats& st = h->stats;
+  std::memset(&st, 0, sizeof(st));
+  st.nnz = nnz;
+  std::vector<int32_t> ident((size_t)M);
+  std::iota(ident.begin(), ident.end(), 0);
+  // DenseRatio of the original order
+  double t0 = now_s();
+  Tiling t_id;
+  tile_rows(A, ident, p->panel_rows, p->dense_min, t_id);
+  st.dense0 = t_id.n_dense();
+  st.t_tile_s += now_s() - t0;
+  bool round1 = p->mode == SR_REORDER_FORCE;
+  if (p->mode == SR_REORDER_AUTO)
+    round1 = !((unsigned __int128)st.dense0 * (uint64_t)p->skip_dense_den >
+               (unsigned __int128)p->skip_dense_num * (uint64_t)nnz);
+  if (round1) {
+    SR_TRY(reorder_round(A.rowptr.data(), A.col.data(), M, *p, s, h->perm1, &st.E1, &st.t_lsh1_s,
+                         &st.t_cluster1_s));
+    t0 = now_s();
+    tile_rows(A, h->perm1, p->panel_rows, p->dense_min, h->tiles);
+    st.t_tile_s += now_s() - t0;
+  } else {
+    h->perm1 = ident;
+    h->tiles = std::move(t_id);
+  }
+  st.round1 = round1 ? 1 : 0;
+  const Tiling& T = h->tiles;
+  st.dense1 = T.n_dense();
+  st.npanels = T.npanels;
+  st.ndense_cols = (int64_t)T.dense_cols.size();
+  for (int64_t q = 0; q < T.npanels; ++q)
+    st.ntiles += (T.dense_ptr[q + 1] - T.dense_ptr[q] + p->tile_cols - 1) / p->tile_cols;
+  avgsim_positions(T, &st.avgsim_num, &st.avgsim_den);
+  bool round2 = p->mode == SR_REORDER_FORCE;
+  if (p->mode == SR_REORDER_AUTO)
+    round2 = !((unsigned __int128)st.avgsim_num * (uint64_t)p->skip_sim_den >
+               (unsigned __int128)p->skip_sim_num * st.avgsim_den);
+  st.round2 = round2 ? 1 : 0;
+  std::vector<int32_t> order;
+  if (round2) {
+    SR_TRY(reorder_round(T.rrow_ptr.data(), T.r_col.data(), M, *p, s, order, &st.E2, &st.t_lsh2_s,
+                         &st.t_cluster2_s));
+  } else {
+    order = ident;
+  }
+  h->perm2.clear();
+  for (int32_t q : order)
+    if (T.rrow_ptr[q + 1] > T.rrow_ptr[q]) h->perm2.push_back(q);
+  st.n_perm2 = (int64_t)h->perm2.size();
+  // shard: contiguous nnz-balanced panel ranges
+  int64_t pb = 0, pe = T.npanels;
+  if (p->world > 1) {
+    std::vector<int64_t> w((size_t)T.npanels), cuts((size_t)p->world + 1);
+    for (int64_t q = 0; q < T.npanels; ++q) {
+      const int64_t a = q * p->panel_rows, b = std::min<int64_t>(M, a + p->panel_rows);
+      w[q] = (T.drow_ptr[b] - T.drow_ptr[a]) + (T.rrow_ptr[b] - T.rrow_ptr[a]);
+    }
+    partition_panels(T.npanels, w.data(), p->world, cuts.data());
+    pb = cuts[p->rank];
+    pe = cuts[p->rank + 1];
+  }
+  st.shard_panel_begin = pb;
+  st.shard_panel_end = pe;
+  SR_TRY(build_exec_plan(h, pb, pe, s));
+  st.shard_nrows = (int64_t)h->shard_rows.size();
+  st.shard_nnz = (int64_t)h->shard_nnz_ids.size();
+  h->reordered = true;
+  st.t_total_s = now_s() - t_start;
+  return SR_OK;
+}
+
+int sr_spmm(sr_csr h, const float* B, int64_t K, int64_t ldb, float* C, int64_t ldc, sr_stream stream) {
+  if (!h) return einval("sr_spmm: NULL handle");
+  if (K < 1 || ldb < K || ldc < K) return einval("sr_spmm: need K >= 1, ldb >= K, ldc >= K");
+  const int64_t rows_out = h->params.world > 1 && h->reordered ? (int64_t)h->shard_rows.size() : h->A.M;
+  if ((rows_out > 0 && !C) || (h->A.nnz() > 0 && !B)) return einval("sr_spmm: NULL operand");
+  if (rows_out == 0) return SR_OK;
+  DeviceGuard dg(h->device);
+  return launch_spmm(h, B, K, ldb, C, ldc, (cudaStream_t)stream, &h->last_launches);
+}
+
+int sr_sddmm(sr_csr h, const float* X, int64_t ldx, const float* Y, int64_t ldy, int64_t K, float* out,
+             sr_stream stream) {
+  if (!h) return einval("sr_sddmm: NULL handle");
+  if (K < 1 || ldx < K || ldy < K) return einval("sr_sddmm: need K >= 1, ldx >= K, ldy >= K");
+  if (h->A.nnz() == 0) return SR_OK;
+  if (!X || !Y || !out) return einval("sr_sddmm: NULL operand");
+  DeviceGuard dg(h->device);
+  return launch_sddmm(h, X, ldx, Y, ldy, K, out, (cudaStream_t)stream, &h->last_launches);
+}
+
+int sr_destroy(sr_csr h) {
+  if (!h) return SR_OK;
+  {
+    DeviceGuard dg(h->device);
+    cudaDeviceSynchronize();
+    if (h->init_stream) cudaStreamDestroy(h->init_stream);
+    delete h;
+  }
+  return SR_OK;
+}
+
+int sr_get_perm(sr_csr h, int which, int32_t* out, int64_t cap, int64_t* len) {
+  if (!h || !len) return einval("sr_get_perm: NULL argument");
+  const std::vector<int32_t>* v = which == 1 ? &h->perm1 : which == 2 ? &h->perm2 : nullptr;
+  if (!v) return einval("sr_get_perm: which must be 1 or 2");
+  *len = (int64_t)v->size();
+  if (cap < *len) return out ? einval("sr_get_perm: capacity too small") : SR_OK;
+  if (out && !v->empty()) std::memcpy(out, v->data(), v->size() * sizeof(int32_t));
+  return SR_OK;
+}
+
+int sr_get_plan_stats(sr_csr h, sr_plan_stats* out) {
+  if (!h || !out) return einval("sr_get_plan_stats: NULL argument");
+  *out = h->stats;
+  return SR_OK;
+}
+
+int sr_export_tiles(sr_csr h, int64_t* dense_ptr, int32_t* dense_cols, int64_t* drow_ptr, int32_t* d_slot,
+                    int64_t* d_pos, int64_t* rrow_ptr, int32_t* r_col, int64_t* r_pos) {
+  if (!h) return einval("sr_export_tiles: NULL handle");
+  if (!h->reordered) {
+    set_error("sr_export_tiles: no plan yet (call sr_reorder)");
+    return SR_ESTATE;
+  }
+  const Tiling& T = h->tiles;
+  const HostCSR& A = h->A;
+  auto orig = [&](int64_t c) -> int64_t { return A.identity_pos ? c : A.opos[c]; };
+  if (dense_ptr) std::copy(T.dense_ptr.begin(), T.dense_ptr.end(), dense_ptr);
+  if (dense_cols) std::copy(T.dense_cols.begin(), T.dense_cols.end(), dense_cols);
+  if (drow_ptr) std::copy(T.drow_ptr.begin(), T.drow_ptr.end(), drow_ptr);
+  if (d_slot) std::copy(T.d_slot.begin(), T.d_slot.end(), d_slot);
+  if (d_pos)
+    for (size_t e = 0; e < T.d_cidx.size(); ++e) d_pos[e] = orig(T.d_cidx[e]);
+  if (rrow_ptr) std::copy(T.rrow_ptr.begin(), T.rrow_ptr.end(), rrow_ptr);
+  if (r_col) std::copy(T.r_col.begin(), T.r_col.end(), r_col);
+  if (r_pos)
+    for (size_t e = 0; e < T.r_cidx.size(); ++e) r_pos[e] = orig(T.r_cidx[e]);
+  return SR_OK;
+}
+
+int sr_shard_rows(sr_csr h, int32_t* rows_out, int64_t cap, int64_t* len) {
+  if (!h || !len) return einval("sr_shard_rows: NULL argument");
+  std::vector<int32_t> all;
+  const std::vector<int32_t>* v = &h->shard_rows;
+  if (!h->reordered) {
+    all = h->perm1;
+    v = &all;
+  }
+  *len = (int64_t)v->size();
+  if (cap < *len) return rows_out ? einval("sr_shard_rows: capacity too small") : SR_OK;
+  if (rows_out && !v->empty()) std::memcpy(rows_out, v->data(), v->size() * sizeof(int32_t));
+  return SR_OK;
+}
+
+int sr_shard_nnz_ids(sr_csr h, int64_t* ids_out, int64_t cap, int64_t* len) {
+  if (!h || !len) return einval("sr_shard_nnz_ids: NULL argument");
+  if (!h->reordered) {
+    set_error("sr_shard_nnz_ids: no plan yet");
+    return SR_ESTATE;
+  }
+  *len = (int64_t)h->shard_nnz_ids.size();
+  if (cap < *len) return ids_out ? einval("sr_shard_nnz_ids: capacity too small") : SR_OK;
+  if (ids_out && *len) std::memcpy(ids_out, h->shard_nnz_ids.data(), *len * sizeof(int64_t));
+  return SR_OK;
+}
+
+int sr_last_launch_count(sr_csr h, int32_t* n) {
+  if (!h || !n) return einval("sr_last_launch_count: NULL argument");
+  *n = h->last_launches;
+  return SR_OK;
+}
+
+int sr_host_cluster(int64_t M, const int64_t* rowptr, const int32_t* colidx, int64_t npairs,
+                    const uint64_t* pairs, const uint32_t* inter, const uint32_t* uni, int32_t threshold_size,
+                    int32_t* perm) {
+  if (M < 0 || !rowptr || !perm || (npairs > 0 && !pairs) || threshold_size < 1)
+    return einval("sr_host_cluster: bad argument");
+  for (int64_t e = 0; e < npairs; ++e) {
+    const uint64_t i = pairs[e] >> 32, j = pairs[e] & 0xFFFFFFFFu;
+    if (i >= j || (int64_t)j >= M || (e > 0 && pairs[e] <= pairs[e - 1]))
+      return einval("sr_host_cluster: pairs must be sorted, unique, i < j < M");
+  }
+  cluster_rows(M, rowptr, colidx, npairs, pairs, inter, uni, threshold_size, perm);
+  return SR_OK;
+}
+
+int sr_host_partition(int64_t npanels, const int64_t* weights, int32_t G, int64_t* cuts) {
+  if (npanels < 0 || G < 1 || !cuts || (npanels > 0 && !weights)) return einval("sr_host_partition: bad argument");
+  partition_panels(npanels, weights, G, cuts);
+  return SR_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,223 @@
+// Host half of the reorder pipeline: Alg 3 clustering and the
+// nnz-balanced panel partition.  The paper runs the clustering on the CPU because it is
+// "inherently sequential, but fast"; so do we.
+//
+// Library design (differs from the oracle's plain heap, same result):
+//  * the initial candidates arrive already sorted in heap order (J desc, then (i, j)
+//    asc; R10) from the GPU, so the initial heap is a read cursor over that array;
+//  * pairs re-inserted by Alg 3 line 28 go to a small binary heap; each pop takes the
+//    larger of the cursor head and the heap top under the same total order;
+//  * candidate-pair membership (line 27, R9) is an open-addressing hash set.
+// Readings R3-R12 decide everything the paper leaves open.
+#include <algorithm>
+#include <cstring>
+#include <numeric>
+#include <queue>
+#include <vector>
+
+#include "internal.h"
+
+namespace sr {
+namespace {
+
+struct Cand {
+  uint32_t inter, uni;
+  uint32_t i, j;  // i < j
+};
+
+// true if a comes before b in heap order (a has higher priority)
+inline bool before(const Cand& a, const Cand& b) {
+  const uint64_t l = (uint64_t)a.inter * b.uni, r = (uint64_t)b.inter * a.uni;
+  if (l != r) return l > r;
+  if (a.i != b.i) return a.i < b.i;
+  return a.j < b.j;
+}
+
+struct AfterCmp {  // std::priority_queue wants "less" = lower priority
+  bool operator()(const Cand& a, const Cand& b) const { return before(b, a); }
+};
+
+class PairSet {
+ public:
+  explicit PairSet(size_t expected) {
+    size_t cap = 16;
+    while (cap < 2 * expected + 16) cap <<= 1;
+    slots_.assign(cap, kEmpty);
+    mask_ = cap - 1;
+  }
+  bool contains(uint64_t k) const {
+    size_t h = hash(k) & mask_;
+    while (true) {
+      const uint64_t v = slots_[h];
+      if (v == k) return true;
+      if (v == kEmpty) return false;
+      h = (h + 1) & mask_;
+    }
+  }
+  void insert(uint64_t k) {
+    if (2 * (size_ + 1) > slots_.size()) grow();
+    size_t h = hash(k) & mask_;
+    while (slots_[h] != kEmpty) {
+      if (slots_[h] == k) return;
+      h = (h + 1) & mask_;
+    }
+    slots_[h] = k;
+    ++size_;
+  }
+
+ private:
+  static constexpr uint64_t kEmpty = ~0ull;
+  static size_t hash(uint64_t k) {
+    k ^= k >> 33;
+    k *= 0xff51afd7ed558ccdull;
+    k ^= k >> 33;
+    k *= 0xc4ceb9fe1a85ec53ull;
+    k ^= k >> 33;
+    return (size_t)k;
+  }
+  void grow() {
+    std::vector<uint64_t> old;
+    old.swap(slots_);
+    slots_.assign(old.size() * 2, kEmpty);
+    mask_ = slots_.size() - 1;
+    size_ = 0;
+    for (uint64_t v : old)
+      if (v != kEmpty) insert(v);
+  }
+  std::vector<uint64_t> slots_;
+  size_t mask_ = 0, size_ = 0;
+};
+
+inline void intersect(const int64_t* rowptr, const int32_t* col, int64_t a, int64_t b,
+                      uint32_t* inter, uint32_t* uni) {
+  const int32_t *p = col + rowptr[a], *pe = col + rowptr[a + 1];
+  const int32_t *q = col + rowptr[b], *qe = col + rowptr[b + 1];
+  const int64_t na = pe - p, nb = qe - q;
+  int64_t n = 0;
+  while (p < pe && q < qe) {
+    const int32_t x = *p, y = *q;
+    n += (x == y);
+    p += (x <= y);
+    q += (y <= x);
+  }
+  *inter = (uint32_t)n;
+  *uni = (uint32_t)(na + nb - n);
+}
+
+}  // namespace
+
+void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t npairs,
+                  const uint64_t* pairs, const uint32_t* inter, const uint32_t* uni,
+                  int32_t threshold_size, int32_t* perm) {
+  // initial candidates in heap order
+  std::vector<Cand> init((size_t)npairs);
+  PairSet members((size_t)npairs + (size_t)npairs / 4);
+  for (int64_t e = 0; e < npairs; ++e) {
+    Cand c;
+    c.i = (uint32_t)(pairs[e] >> 32);
+    c.j = (uint32_t)(pairs[e] & 0xFFFFFFFFu);
+    if (inter) {
+      c.inter = inter[e];
+      c.uni = uni[e];
+    } else {
+      intersect(rowptr, col, c.i, c.j, &c.inter, &c.uni);
+    }
+    if (c.uni == 0) c.uni = 1;  // J(empty, empty) := 0/1 (R16)
+    init[e] = c;
+    members.insert(pairs[e]);
+  }
+  bool sorted = true;
+  for (int64_t e = 1; e < npairs && sorted; ++e) sorted = !before(init[e], init[e - 1]);
+  if (!sorted) std::stable_sort(init.begin(), init.end(), before);
+
+  std::vector<int32_t> cid((size_t)M), csz((size_t)M, 1);
+  std::vector<uint8_t> dead((size_t)M, 0);
+  std::iota(cid.begin(), cid.end(), 0);
+  auto root = [&](int32_t x) {  // path halving
+    while (x != cid[x]) {
+      cid[x] = cid[cid[x]];
+      x = cid[x];
+    }
+    return x;
+  };
+  std::priority_queue<Cand, std::vector<Cand>, AfterCmp> extra;
+  size_t cur = 0;
+  int64_t nclusters = M;
+  while ((cur < init.size() || !extra.empty()) && nclusters > 0) {
+    Cand top;
+    if (cur < init.size() && (extra.empty() || before(init[cur], extra.top()))) {
+      top = init[cur++];
+    } else {
+      top = extra.top();
+      extra.pop();
+    }
+    int32_t i = (int32_t)top.i, j = (int32_t)top.j;
+    if (cid[i] == i && cid[j] == j) {
+      if (dead[i] || dead[j]) continue;
+      // the larger cluster absorbs the smaller; equal sizes: smaller index (R6)
+      const bool i_wins = csz[i] > csz[j] || (csz[i] == csz[j] && i < j);
+      const int32_t w = i_wins ? i : j, l = i_wins ? j : i;
+      cid[l] = w;
+      csz[w] += csz[l];  // R4
+      --nclusters;
+      if (csz[w] >= threshold_size) {  // R7, R5
+        dead[w] = 1;
+        --nclusters;
+      }
+    } else {
+      i = root(i);
+      j = root(j);
+      if (dead[i] || dead[j] || i == j) continue;
+      const uint32_t lo = (uint32_t)std::min(i, j), hi = (uint32_t)std::max(i, j);
+      const uint64_t key = ((uint64_t)lo << 32) | hi;
+      if (members.contains(key)) continue;
+      Cand c;
+      c.i = lo;
+      c.j = hi;
+      intersect(rowptr, col, lo, hi, &c.inter, &c.uni);  // representing rows (R8)
+      if (c.uni == 0) c.uni = 1;
+      extra.push(c);
+      members.insert(key);
+    }
+  }
+  // rule B (R11): clusters of >= 2 rows by ascending root, then singletons ascending
+  std::vector<int32_t> r_of((size_t)M);
+  std::vector<int64_t> count((size_t)M + 1, 0);
+  for (int64_t x = 0; x < M; ++x) {
+    r_of[x] = root((int32_t)x);
+    ++count[r_of[x]];
+  }
+  // offsets: cluster roots ascending, members ascending (counting sort by root)
+  std::vector<int64_t> off((size_t)M, 0);
+  int64_t pos = 0;
+  for (int64_t r = 0; r < M; ++r)
+    if (count[r] >= 2) {
+      off[r] = pos;
+      pos += count[r];
+    }
+  int64_t spos = pos;
+  for (int64_t x = 0; x < M; ++x) {
+    const int32_t r = r_of[x];
+    if (count[r] >= 2)
+      perm[off[r]++] = (int32_t)x;
+    else
+      perm[spos++] = (int32_t)x;
+  }
+}
+
+void partition_panels(int64_t npanels, const int64_t* w, int32_t G, int64_t* cuts) {
+  std::vector<int64_t> prefix((size_t)npanels + 1, 0);
+  for (int64_t p = 0; p < npanels; ++p) prefix[p + 1] = prefix[p] + w[p];
+  const int64_t total = prefix[npanels];
+  cuts[0] = 0;
+  cuts[G] = npanels;
+  for (int32_t g = 1; g < G; ++g) {
+    // smallest p with prefix[p]·G >= g·total  (prefix is non-decreasing)
+    auto it = std::partition_point(prefix.begin(), prefix.end(), [&](int64_t v) {
+      return (unsigned __int128)v * (unsigned)G < (unsigned __int128)g * (uint64_t)total;
+    });
+    cuts[g] = std::min<int64_t>(it - prefix.begin(), npanels);
+  }
+}
+
+}  // namespace sr

@@ -1,0 +1,599 @@
+// sm_100a SpMM / SDDMM execution over an ASpT plan (Alg 1, Alg 2
+// P:78-92, row-wise GPU mapping P:101, adaptive sparse tiling P:111, Fig 5).
+//
+// Phase D ("dense tiles"): one CTA per row panel that has dense columns.  The B/Y
+//   rows of the panel's dense columns are staged into shared memory tile by tile with
+//   bulk asynchronous copies (cp.async.bulk -> UBLKCP, completion on an mbarrier with
+//   transaction counts), double-buffered so tile t+1 streams in while tile t is used.
+//   Warp w owns panel rows w, w+W, ...; each dense nnz is served from shared memory.
+// Phase S ("sparse remainder"): one warp per work item = a remainder row
+//   in round-2 order (perm2) or a bounded chunk of a long row; lanes own 16-byte column
+//   fragments, so every gathered B/Y row is one coalesced 128-bit load per lane; U gathers
+//   are in flight per lane.  SDDMM reduces each dot product with warp shuffles.
+// Lane geometry: LPG lanes cover LPG·VEC columns of one nnz; G = 32/LPG groups of a warp
+//   work on G different nnz at once (K = 32 -> 4 nnz per warp instruction).
+#include <algorithm>
+
+#include "internal.h"
+
+namespace sr {
+namespace {
+
+constexpr unsigned FULL = 0xffffffffu;
+
+template <int VEC>
+struct Frag;
+template <>
+struct Frag<4> {
+  float4 v;
+  __device__ __forceinline__ void zero() { v = make_float4(0.f, 0.f, 0.f, 0.f); }
+  __device__ __forceinline__ void load_g(const float* p) { v = __ldg(reinterpret_cast<const float4*>(p)); }
+  __device__ __forceinline__ void load_cg(const float* p) { v = __ldcg(reinterpret_cast<const float4*>(p)); }
+  __device__ __forceinline__ void load_s(const float* p) { v = *reinterpret_cast<const float4*>(p); }
+  __device__ __forceinline__ void fma(float a, const Frag& b) {
+    v.x = fmaf(a, b.v.x, v.x); v.y = fmaf(a, b.v.y, v.y);
+    v.z = fmaf(a, b.v.z, v.z); v.w = fmaf(a, b.v.w, v.w);
+  }
+  __device__ __forceinline__ void add(const Frag& b) { v.x += b.v.x; v.y += b.v.y; v.z += b.v.z; v.w += b.v.w; }
+  __device__ __forceinline__ float dot(const Frag& b) const {
+    return fmaf(v.x, b.v.x, fmaf(v.y, b.v.y, fmaf(v.z, b.v.z, v.w * b.v.w)));
+  }
+  __device__ __forceinline__ void xor_add(int off) {
+    v.x += __shfl_xor_sync(FULL, v.x, off); v.y += __shfl_xor_sync(FULL, v.y, off);
+    v.z += __shfl_xor_sync(FULL, v.z, off); v.w += __shfl_xor_sync(FULL, v.w, off);
+  }
+  __device__ __forceinline__ void store(float* p) const { *reinterpret_cast<float4*>(p) = v; }
+  __device__ __forceinline__ void store_cs(float* p) const { __stcs(reinterpret_cast<float4*>(p), v); }
+};
+template <>
+struct Frag<1> {
+  float v;
+  __device__ __forceinline__ void zero() { v = 0.f; }
+  __device__ __forceinline__ void load_g(const float* p) { v = __ldg(p); }
+  __device__ __forceinline__ void load_cg(const float* p) { v = __ldcg(p); }
+  __device__ __forceinline__ void load_s(const float* p) { v = *p; }
+  __device__ __forceinline__ void fma(float a, const Frag& b) { v = fmaf(a, b.v, v); }
+  __device__ __forceinline__ void add(const Frag& b) { v += b.v; }
+  __device__ __forceinline__ float dot(const Frag& b) const { return v * b.v; }
+  __device__ __forceinline__ void xor_add(int off) { v += __shfl_xor_sync(FULL, v, off); }
+  __device__ __forceinline__ void store(float* p) const { *p = v; }
+  __device__ __forceinline__ void store_cs(float* p) const { __stcs(p, v); }
+};
+
+// ------------------------------------------------------------------ mbarrier / bulk copy
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P1;\n\t"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n\t"
+      "@!P1 bra WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+// ------------------------------------------------------------------ phase S: SpMM
+template <int LPG, int VEC, int U>
+__global__ void __launch_bounds__(256) spmm_sparse_kernel(
+    const Item* __restrict__ items, const uint32_t* __restrict__ meta, int64_t n_items,
+    const int2* __restrict__ ent, const float* __restrict__ B, int64_t ldb, float* __restrict__ C,
+    int64_t ldc, int K, float* __restrict__ scratch, const int2* __restrict__ split_info,
+    int* __restrict__ split_counter) {
+  constexpr int G = 32 / LPG;
+  constexpr int KC = LPG * VEC;
+  const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
+  const int64_t it = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  if (it >= n_items) return;
+  const Item item = items[it];
+  const uint32_t mt = meta[it];
+  for (int k0 = 0; k0 < K; k0 += KC) {
+    const int kk = k0 + lg * VEC;
+    const bool kv = kk < K;
+    Frag<VEC> acc;
+    acc.zero();
+    for (int e = item.e0; e < item.e1; e += 32) {
+      const int n = min(32, item.e1 - e);
+      const int2 my = lane < n ? __ldcs(ent + e + lane) : make_int2(0, 0);
+      for (int base = 0; base < n; base += G * U) {
+        Frag<VEC> b[U];
+        float a[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const int j = base + u * G + g;
+          const int src = j & 31;
+          const int c = __shfl_sync(FULL, my.x, src);
+          const float v = __int_as_float(__shfl_sync(FULL, my.y, src));
+          const bool ok = (j < n) && kv;
+          a[u] = ok ? v : 0.f;
+          if (ok) b[u].load_g(B + (int64_t)c * ldb + kk); else b[u].zero();
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) acc.fma(a[u], b[u]);
+      }
+    }
+#pragma unroll
+    for (int off = LPG; off < 32; off <<= 1) acc.xor_add(off);
+    if (g == 0 && kv) {
+      if (mt & kItemSplit) {
+        acc.store(scratch + (int64_t)(mt & kItemSlotMask) * K + kk);
+      } else {
+        float* dst = C + (int64_t)item.out * ldc + kk;
+        if (mt & kItemRMW) {
+          Frag<VEC> old;
+          old.load_cg(dst);
+          acc.add(old);
+        }
+        acc.store_cs(dst);
+      }
+    }
+  }
+  if (mt & kItemSplit) {
+    // deterministic combine: the last chunk to finish sums all chunk partials in order
+    __threadfence();
+    __syncwarp();
+    const int slot = (int)(mt & kItemSlotMask);
+    const int2 si = split_info[slot];
+    int last = 0;
+    if (lane == 0) last = (atomicAdd(split_counter + si.x, 1) == si.y - 1);
+    last = __shfl_sync(FULL, last, 0);
+    if (last) {
+      __threadfence();
+      for (int k = lane * VEC; k < K; k += 32 * VEC) {
+        Frag<VEC> s;
+        s.zero();
+        for (int c = 0; c < si.y; ++c) {
+          Frag<VEC> part;
+          part.load_cg(scratch + (int64_t)(si.x + c) * K + k);
+          s.add(part);
+        }
+        float* dst = C + (int64_t)item.out * ldc + k;
+        if (mt & kItemRMW) {
+          Frag<VEC> old;
+          old.load_cg(dst);
+          s.add(old);
+        }
+        s.store_cs(dst);
+      }
+      if (lane == 0) split_counter[si.x] = 0;
+    }
+  }
+}
+
+// ------------------------------------------------------------------ phase S: SDDMM
+template <int LPG, int VEC, int U, int NCH>
+__global__ void __launch_bounds__(256) sddmm_sparse_kernel(
+    const Item* __restrict__ items, int64_t n_items, const int2* __restrict__ ent,
+    const int32_t* __restrict__ oidx, const float* __restrict__ X, int64_t ldx,
+    const float* __restrict__ Y, int64_t ldy, int K, float* __restrict__ out) {
+  constexpr int G = 32 / LPG;
+  constexpr int KC = LPG * VEC;
+  const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
+  const int64_t it = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  if (it >= n_items) return;
+  const Item item = items[it];
+  Frag<VEC> x[NCH];
+#pragma unroll
+  for (int c = 0; c < NCH; ++c) {
+    const int kk = c * KC + lg * VEC;
+    if (kk < K) x[c].load_g(X + (int64_t)item.xrow * ldx + kk); else x[c].zero();
+  }
+  for (int e = item.e0; e < item.e1; e += 32) {
+    const int n = min(32, item.e1 - e);
+    const int2 my = lane < n ? __ldcs(ent + e + lane) : make_int2(0, 0);
+    const int myo = lane < n ? __ldcs(oidx + e + lane) : 0;
+    for (int base = 0; base < n; base += G * U) {
+      float part[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int j = base + u * G + g;
+        const int c = __shfl_sync(FULL, my.x, j & 31);
+        const bool ok = j < n;
+        float d = 0.f;
+#pragma unroll
+        for (int ch = 0; ch < NCH; ++ch) {
+          const int kk = ch * KC + lg * VEC;
+          if (ok && kk < K) {
+            Frag<VEC> y;
+            y.load_g(Y + (int64_t)c * ldy + kk);
+            d += x[ch].dot(y);
+          }
+        }
+        part[u] = d;
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+#pragma unroll
+        for (int off = LPG / 2; off > 0; off >>= 1) part[u] += __shfl_xor_sync(FULL, part[u], off);
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int j = base + u * G + g;
+        const float v = __int_as_float(__shfl_sync(FULL, my.y, j & 31));
+        const int o = __shfl_sync(FULL, myo, j & 31);
+        if (lg == 0 && j < n) __stcs(out + o, v * part[u]);
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------ phase D
+constexpr int kDenseWarps = 8;  // phase-D CTA = 8 warps; RPW = panel rows per warp (8 or 16)
+
+// SpMM dense tiles.  Dynamic smem: 2 stages × SW slots × KC floats.
+template <int LPG, int VEC, int U, int kRPW, bool kBulk>
+__global__ void __launch_bounds__(256, 1) spmm_dense_kernel(
+    const DPanel* __restrict__ panels, const int32_t* __restrict__ dense_cols,
+    const int32_t* __restrict__ drow_ptr, const int2* __restrict__ d_ent,
+    const int32_t* __restrict__ pos_out, const float* __restrict__ B, int64_t ldb,
+    float* __restrict__ C, int64_t ldc, int K, int SW) {
+  constexpr int G = 32 / LPG;
+  constexpr int KC = LPG * VEC;
+  extern __shared__ __align__(128) float smem[];
+  __shared__ uint64_t full[2];
+  const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
+  const int warp = threadIdx.x >> 5, W = blockDim.x >> 5;
+  const DPanel pn = panels[blockIdx.x];
+  const int nd = pn.dc1 - pn.dc0;
+  const int ntile = (nd + SW - 1) / SW;
+  if (kBulk && threadIdx.x == 0) {
+    mbar_init(&full[0], 1);
+    mbar_init(&full[1], 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  int tcount = 0;  // tiles issued so far (stage = tcount & 1, parity = (tcount >> 1) & 1)
+  for (int k0 = 0; k0 < K; k0 += KC) {
+    const int kw = min(KC, K - k0);  // columns staged per slot
+    auto issue = [&](int t, int st) {
+      const int s0 = t * SW, ns = min(SW, nd - s0);
+      float* dst = smem + (size_t)st * SW * KC;
+      if (kBulk) {
+        if (warp == 0) {
+          if (lane == 0) mbar_expect_tx(&full[st], (uint32_t)(ns * kw * 4));
+          __syncwarp();
+          for (int j = lane; j < ns; j += 32)
+            bulk_g2s(dst + (size_t)j * KC, B + (int64_t)dense_cols[pn.dc0 + s0 + j] * ldb + k0,
+                     (uint32_t)(kw * 4), &full[st]);
+        }
+      } else {
+        for (int idx = threadIdx.x; idx < ns * kw; idx += blockDim.x) {
+          const int j = idx / kw, k = idx % kw;
+          dst[(size_t)j * KC + k] = __ldg(B + (int64_t)dense_cols[pn.dc0 + s0 + j] * ldb + k0 + k);
+        }
+      }
+    };
+    int cur[kRPW], end[kRPW];
+    bool has[kRPW];
+    Frag<VEC> acc[kRPW];
+#pragma unroll
+    for (int i = 0; i < kRPW; ++i) {
+      const int r = warp + i * W;
+      if (r < pn.nrows) {
+        cur[i] = drow_ptr[pn.q0 + r];
+        end[i] = drow_ptr[pn.q0 + r + 1];
+      } else {
+        cur[i] = end[i] = 0;
+      }
+      has[i] = end[i] > cur[i];
+      acc[i].zero();
+    }
+    const int kk = k0 + lg * VEC;
+    const bool kv = kk < K;
+    if (ntile > 0) issue(0, tcount & 1);
+    for (int t = 0; t < ntile; ++t) {
+      const int st = (tcount + t) & 1;
+      if (t + 1 < ntile) issue(t + 1, (tcount + t + 1) & 1);
+      if (kBulk) mbar_wait(&full[st], ((tcount + t) >> 1) & 1);
+      else __syncthreads();
+      const float* tile = smem + (size_t)st * SW * KC;
+      const int s_lo = t * SW, s_hi = s_lo + SW;
+#pragma unroll
+      for (int i = 0; i < kRPW; ++i) {
+        while (cur[i] < end[i]) {
+          const int navail = min(32, end[i] - cur[i]);
+          const int2 my = lane < navail ? d_ent[cur[i] + lane] : make_int2(0x7fffffff, 0);
+          const unsigned inside = __ballot_sync(FULL, lane < navail && my.x < s_hi);
+          const int n = __popc(inside);
+          for (int base = 0; base < n; base += G * U) {
+            Frag<VEC> b[U];
+            float a[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+              const int j = base + u * G + g;
+              const int slot = __shfl_sync(FULL, my.x, j & 31);
+              const float v = __int_as_float(__shfl_sync(FULL, my.y, j & 31));
+              const bool ok = j < n && kv;
+              a[u] = ok ? v : 0.f;
+              if (ok) b[u].load_s(tile + (size_t)(slot - s_lo) * KC + lg * VEC); else b[u].zero();
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) acc[i].fma(a[u], b[u]);
+          }
+          cur[i] += n;
+          if (n < navail) break;
+        }
+      }
+      __syncthreads();  // stage st may be overwritten by the next issue
+    }
+    tcount += ntile;
+#pragma unroll
+    for (int i = 0; i < kRPW; ++i) {
+#pragma unroll
+      for (int off = LPG; off < 32; off <<= 1) acc[i].xor_add(off);
+      const int r = warp + i * W;
+      if (has[i] && g == 0 && kv) acc[i].store_cs(C + (int64_t)pos_out[pn.q0 + r] * ldc + kk);
+    }
+  }
+}
+
+// SDDMM dense tiles.  Slots hold the full (padded) K of each Y row: NCH × KC floats.
+template <int LPG, int VEC, int U, int NCH, int kRPW, bool kBulk>
+__global__ void __launch_bounds__(256, 1) sddmm_dense_kernel(
+    const DPanel* __restrict__ panels, const int32_t* __restrict__ dense_cols,
+    const int32_t* __restrict__ drow_ptr, const int2* __restrict__ d_ent,
+    const int32_t* __restrict__ d_oidx, const int32_t* __restrict__ pos_xrow,
+    const float* __restrict__ X, int64_t ldx, const float* __restrict__ Y, int64_t ldy, int K,
+    int SW, float* __restrict__ out) {
+  constexpr int G = 32 / LPG;
+  constexpr int KC = LPG * VEC;
+  constexpr int SLOT = NCH * KC;
+  extern __shared__ __align__(128) float smem[];
+  __shared__ uint64_t full[2];
+  const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
+  const int warp = threadIdx.x >> 5, W = blockDim.x >> 5;
+  const DPanel pn = panels[blockIdx.x];
+  const int nd = pn.dc1 - pn.dc0;
+  const int ntile = (nd + SW - 1) / SW;
+  if (kBulk && threadIdx.x == 0) {
+    mbar_init(&full[0], 1);
+    mbar_init(&full[1], 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  auto issue = [&](int t, int st) {
+    const int s0 = t * SW, ns = min(SW, nd - s0);
+    float* dst = smem + (size_t)st * SW * SLOT;
+    if (kBulk) {
+      if (warp == 0) {
+        if (lane == 0) mbar_expect_tx(&full[st], (uint32_t)(ns * K * 4));
+        __syncwarp();
+        for (int j = lane; j < ns; j += 32)
+          bulk_g2s(dst + (size_t)j * SLOT, Y + (int64_t)dense_cols[pn.dc0 + s0 + j] * ldy,
+                   (uint32_t)(K * 4), &full[st]);
+      }
+    } else {
+      for (int idx = threadIdx.x; idx < ns * K; idx += blockDim.x) {
+        const int j = idx / K, k = idx % K;
+        dst[(size_t)j * SLOT + k] = __ldg(Y + (int64_t)dense_cols[pn.dc0 + s0 + j] * ldy + k);
+      }
+    }
+  };
+  int cur[kRPW], end[kRPW];
+#pragma unroll
+  for (int i = 0; i < kRPW; ++i) {
+    const int r = warp + i * W;
+    if (r < pn.nrows) {
+      cur[i] = drow_ptr[pn.q0 + r];
+      end[i] = drow_ptr[pn.q0 + r + 1];
+    } else {
+      cur[i] = end[i] = 0;
+    }
+  }
+  if (ntile > 0) issue(0, 0);
+  for (int t = 0; t < ntile; ++t) {
+    const int st = t & 1;
+    if (t + 1 < ntile) issue(t + 1, (t + 1) & 1);
+    if (kBulk) mbar_wait(&full[st], (t >> 1) & 1);
+    else __syncthreads();
+    const float* tile = smem + (size_t)st * SW * SLOT;
+    const int s_lo = t * SW, s_hi = s_lo + SW;
+#pragma unroll
+    for (int i = 0; i < kRPW; ++i) {
+      if (cur[i] >= end[i]) continue;
+      const int r = warp + i * W;
+      const int xr = pos_xrow[pn.q0 + r];
+      Frag<VEC> x[NCH];
+#pragma unroll
+      for (int c = 0; c < NCH; ++c) {
+        const int kk = c * KC + lg * VEC;
+        if (kk < K) x[c].load_g(X + (int64_t)xr * ldx + kk); else x[c].zero();
+      }
+      while (cur[i] < end[i]) {
+        const int navail = min(32, end[i] - cur[i]);
+        const int2 my = lane < navail ? d_ent[cur[i] + lane] : make_int2(0x7fffffff, 0);
+        const int myo = lane < navail ? d_oidx[cur[i] + lane] : 0;
+        const unsigned inside = __ballot_sync(FULL, lane < navail && my.x < s_hi);
+        const int n = __popc(inside);
+        for (int base = 0; base < n; base += G * U) {
+          float part[U];
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            const int j = base + u * G + g;
+            const int slot = __shfl_sync(FULL, my.x, j & 31);
+            float d = 0.f;
+            if (j < n) {
+#pragma unroll
+              for (int c = 0; c < NCH; ++c) {
+                const int kk = c * KC + lg * VEC;
+                if (kk < K) {
+                  Frag<VEC> y;
+                  y.load_s(tile + (size_t)(slot - s_lo) * SLOT + kk);
+                  d += x[c].dot(y);
+                }
+              }
+            }
+            part[u] = d;
+          }
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+#pragma unroll
+            for (int off = LPG / 2; off > 0; off >>= 1) part[u] += __shfl_xor_sync(FULL, part[u], off);
+          }
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            const int j = base + u * G + g;
+            const float v = __int_as_float(__shfl_sync(FULL, my.y, j & 31));
+            const int o = __shfl_sync(FULL, myo, j & 31);
+            if (lg == 0 && j < n) __stcs(out + o, v * part[u]);
+          }
+        }
+        cur[i] += n;
+        if (n < navail) break;
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// ------------------------------------------------------------------ host dispatch
+inline int next_pow2(int x) {
+  int p = 1;
+  while (p < x) p <<= 1;
+  return p;
+}
+
+constexpr int kStageBytes = 48 * 1024;
+constexpr int kSparseWarps = 8;
+
+template <int LPG, int VEC>
+int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int64_t ldc,
+             cudaStream_t s, int32_t* launches) {
+  DevPlan& P = h->plan;
+  constexpr int KC = LPG * VEC;
+  constexpr int U = (LPG == 32) ? 8 : 4;  // gathers in flight per lane (phase S)
+  constexpr int UD = 4;                   // shared-memory reads in flight per lane (phase D)
+  if (P.n_dpanels > 0) {
+    const int SW = std::max(1, std::min(P.tile_cols, kStageBytes / (KC * 4)));
+    const size_t smem = (size_t)2 * SW * KC * sizeof(float);
+    auto launch = [&](auto kern) -> int {
+      SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+      kern<<<(unsigned)P.n_dpanels, kDenseWarps * 32, smem, s>>>(P.dpanels.p, P.dense_cols.p, P.drow_ptr.p,
+                                                                P.d_ent.p, P.pos_out.p, B, ldb, C, ldc, (int)K, SW);
+      SR_CUDA_TRY(cudaGetLastError());
+      return SR_OK;
+    };
+    if (VEC == 4) {
+      if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 8, true>));
+      else SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 16, true>));
+    } else {
+      SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 16, false>));
+    }
+    ++*launches;
+  }
+  if (P.n_items > 0) {
+    if (P.n_slots > 0 && P.scratch_k < K) {
+      SR_TRY(P.scratch.alloc((size_t)P.n_slots * K));
+      P.scratch_k = K;
+    }
+    const unsigned grid = (unsigned)((P.n_items + kSparseWarps - 1) / kSparseWarps);
+    spmm_sparse_kernel<LPG, VEC, U><<<grid, kSparseWarps * 32, 0, s>>>(
+        P.items.p, P.item_meta.p, P.n_items, P.s_ent.p, B, ldb, C, ldc, (int)K, P.scratch.p,
+        P.split_info.p, P.split_counter.p);
+    SR_CUDA_TRY(cudaGetLastError());
+    ++*launches;
+  }
+  return SR_OK;
+}
+
+template <int LPG, int VEC, int NCH>
+int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t ldy, int64_t K,
+              float* out, cudaStream_t s, int32_t* launches) {
+  DevPlan& P = h->plan;
+  constexpr int KC = LPG * VEC;
+  constexpr int U = (LPG == 32) ? 4 : 2;
+  if (P.n_dpanels > 0) {
+    const int slot_floats = NCH * KC;
+    const int SW = std::max(1, std::min(P.tile_cols, kStageBytes / (slot_floats * 4)));
+    const size_t smem = (size_t)2 * SW * slot_floats * sizeof(float);
+    auto launch = [&](auto kern) -> int {
+      SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+      kern<<<(unsigned)P.n_dpanels, kDenseWarps * 32, smem, s>>>(P.dpanels.p, P.dense_cols.p, P.drow_ptr.p,
+                                                                P.d_ent.p, P.d_oidx.p, P.pos_xrow.p, X, ldx, Y,
+                                                                ldy, (int)K, SW, out);
+      SR_CUDA_TRY(cudaGetLastError());
+      return SR_OK;
+    };
+    if (VEC == 4) {
+      if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, U, NCH, 8, true>));
+      else SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, U, NCH, 16, true>));
+    } else {
+      SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, U, NCH, 16, false>));
+    }
+    ++*launches;
+  }
+  if (P.n_sitems > 0) {
+    const unsigned grid = (unsigned)((P.n_sitems + kSparseWarps - 1) / kSparseWarps);
+    sddmm_sparse_kernel<LPG, VEC, U, NCH><<<grid, kSparseWarps * 32, 0, s>>>(
+        P.items.p, P.n_sitems, P.s_ent.p, P.s_oidx.p, X, ldx, Y, ldy, (int)K, out);
+    SR_CUDA_TRY(cudaGetLastError());
+    ++*launches;
+  }
+  return SR_OK;
+}
+
+}  // namespace
+
+int launch_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int64_t ldc,
+                cudaStream_t s, int32_t* launches) {
+  *launches = 0;
+  const bool vec = (K % 4 == 0) && (ldb % 4 == 0) && (ldc % 4 == 0) &&
+                   ((uintptr_t)B % 16 == 0) && ((uintptr_t)C % 16 == 0);
+  const int VEC = vec ? 4 : 1;
+  const int lpg = std::min(32, next_pow2((int)std::min<int64_t>(32, (K + VEC - 1) / VEC)));
+#define SR_S(L, V) return run_spmm<L, V>(h, B, K, ldb, C, ldc, s, launches)
+  if (vec) {
+    switch (lpg) { case 1: SR_S(1, 4); case 2: SR_S(2, 4); case 4: SR_S(4, 4); case 8: SR_S(8, 4); case 16: SR_S(16, 4); default: SR_S(32, 4); }
+  } else {
+    switch (lpg) { case 1: SR_S(1, 1); case 2: SR_S(2, 1); case 4: SR_S(4, 1); case 8: SR_S(8, 1); case 16: SR_S(16, 1); default: SR_S(32, 1); }
+  }
+#undef SR_S
+}
+
+int launch_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t ldy, int64_t K,
+                 float* out, cudaStream_t s, int32_t* launches) {
+  *launches = 0;
+  const bool vec = (K % 4 == 0) && (ldx % 4 == 0) && (ldy % 4 == 0) &&
+                   ((uintptr_t)X % 16 == 0) && ((uintptr_t)Y % 16 == 0);
+  const int VEC = vec ? 4 : 1;
+  const int lpg = std::min(32, next_pow2((int)std::min<int64_t>(32, (K + VEC - 1) / VEC)));
+  const int64_t KC = (int64_t)lpg * VEC;
+  const int64_t nch = (K + KC - 1) / KC;
+  if (nch > 8) {
+    set_error("sr_sddmm: K too large (max 1024 on the vector path, 256 on the scalar path)");
+    return SR_EUNSUPPORTED;
+  }
+#define SR_D(L, V, N) return run_sddmm<L, V, N>(h, X, ldx, Y, ldy, K, out, s, launches)
+  if (vec) {
+    if (lpg < 32) {
+      switch (lpg) { case 1: SR_D(1, 4, 1); case 2: SR_D(2, 4, 1); case 4: SR_D(4, 4, 1); case 8: SR_D(8, 4, 1); default: SR_D(16, 4, 1); }
+    }
+    switch (nch) { case 1: SR_D(32, 4, 1); case 2: SR_D(32, 4, 2); case 3: case 4: SR_D(32, 4, 4); default: SR_D(32, 4, 8); }
+  } else {
+    if (lpg < 32) {
+      switch (lpg) { case 1: SR_D(1, 1, 1); case 2: SR_D(2, 1, 1); case 4: SR_D(4, 1, 1); case 8: SR_D(8, 1, 1); default: SR_D(16, 1, 1); }
+    }
+    switch (nch) { case 1: SR_D(32, 1, 1); case 2: SR_D(32, 1, 2); case 3: case 4: SR_D(32, 1, 4); default: SR_D(32, 1, 8); }
+  }
+#undef SR_D
+}
+
+}  // namespace sr

@@ -1,0 +1,178 @@
+// Internal declarations of libsr (the product library).  Shares nothing with oracle/.
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/sr.h"
+
+namespace sr {
+
+void set_error(const std::string& msg);
+
+struct Status {
+  int code = SR_OK;
+  static Status ok() { return Status(); }
+};
+
+#define SR_CUDA_TRY(expr)                                                              \
+  do {                                                                                 \
+    cudaError_t _e = (expr);                                                           \
+    if (_e != cudaSuccess) {                                                           \
+      ::sr::set_error(std::string(#expr) + ": " + cudaGetErrorString(_e));             \
+      return SR_ECUDA;                                                                 \
+    }                                                                                  \
+  } while (0)
+
+#define SR_TRY(expr)        \
+  do {                      \
+    int _rc = (expr);       \
+    if (_rc != SR_OK) return _rc; \
+  } while (0)
+
+// RAII device buffer
+template <typename T>
+struct DevBuf {
+  T* p = nullptr;
+  size_t n = 0;
+  DevBuf() = default;
+  DevBuf(const DevBuf&) = delete;
+  DevBuf& operator=(const DevBuf&) = delete;
+  ~DevBuf() { release(); }
+  void release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    n = 0;
+  }
+  int alloc(size_t count) {
+    release();
+    if (count == 0) count = 1;
+    if (cudaMalloc(&p, count * sizeof(T)) != cudaSuccess) {
+      cudaGetLastError();
+      set_error("cudaMalloc of " + std::to_string(count * sizeof(T)) + " bytes failed");
+      p = nullptr;
+      return SR_ENOMEM;
+    }
+    n = count;
+    return SR_OK;
+  }
+  int upload(const T* host, size_t count, cudaStream_t s) {
+    SR_TRY(alloc(count));
+    if (count) SR_CUDA_TRY(cudaMemcpyAsync(p, host, count * sizeof(T), cudaMemcpyHostToDevice, s));
+    return SR_OK;
+  }
+  int upload(const std::vector<T>& v, cudaStream_t s) { return upload(v.data(), v.size(), s); }
+};
+
+// A column-sorted CSR on the host (canonical form of the caller's matrix).
+struct HostCSR {
+  int64_t M = 0, N = 0;
+  std::vector<int64_t> rowptr;  // M+1
+  std::vector<int32_t> col;     // nnz
+  std::vector<float> val;       // nnz
+  std::vector<int32_t> opos;    // nnz: caller's original index of each canonical nnz
+  bool identity_pos = true;
+  int64_t nnz() const { return rowptr.empty() ? 0 : rowptr.back(); }
+};
+
+// ASpT tiling of a row order (host result, positions q = index into perm).
+struct Tiling {
+  int64_t npanels = 0;
+  std::vector<int64_t> dense_ptr;   // npanels+1
+  std::vector<int32_t> dense_cols;  // Σ|D_p|
+  std::vector<int64_t> drow_ptr;    // M+1 over positions
+  std::vector<int32_t> d_slot;      // dense nnz: slot in D_p (ascending per position)
+  std::vector<int64_t> d_cidx;      // dense nnz: canonical nnz index
+  std::vector<int64_t> rrow_ptr;    // M+1 over positions
+  std::vector<int32_t> r_col;       // remainder nnz: column (CSR order)
+  std::vector<int64_t> r_cidx;      // remainder nnz: canonical nnz index
+  int64_t n_dense() const { return drow_ptr.empty() ? 0 : drow_ptr.back(); }
+};
+
+// Phase-S work item: one warp processes entries [e0, e1) of the remainder stream.
+struct __align__(16) Item {
+  int32_t e0, e1;
+  int32_t xrow;  // original row id (X row for SDDMM)
+  int32_t out;   // SpMM output row (original id, or packed shard index)
+};
+
+constexpr uint32_t kItemRMW = 1u << 31;    // C[out] += partial (row also has dense-tile nnz)
+constexpr uint32_t kItemSplit = 1u << 30;  // partial of a split long row -> scratch slot
+constexpr uint32_t kItemSlotMask = (1u << 30) - 1;
+
+// Phase-D work unit: one CTA per panel with at least one dense column.
+struct __align__(16) DPanel {
+  int32_t q0, nrows;  // positions [q0, q0+nrows)
+  int32_t dc0, dc1;   // dense_cols[dc0, dc1) = D_p
+};
+
+// Device-resident execution plan.
+struct DevPlan {
+  // phase D
+  DevBuf<DPanel> dpanels;
+  int64_t n_dpanels = 0;
+  DevBuf<int32_t> dense_cols;
+  DevBuf<int32_t> drow_ptr;   // positions -> offsets into d_ent
+  DevBuf<int2> d_ent;         // {slot, __float_as_int(val)}
+  DevBuf<int32_t> d_oidx;     // SDDMM output index per dense nnz
+  DevBuf<int32_t> pos_xrow;   // position -> original row
+  DevBuf<int32_t> pos_out;    // position -> SpMM output row
+  // phase S
+  DevBuf<int2> s_ent;         // {col, __float_as_int(val)} remainder stream
+  DevBuf<int32_t> s_oidx;     // SDDMM output index per remainder nnz
+  DevBuf<Item> items;         // SpMM items (remainder rows, split chunks, zero rows)
+  DevBuf<uint32_t> item_meta;
+  int64_t n_items = 0;
+  DevBuf<Item> sitems;        // SDDMM items (remainder rows / chunks only)
+  int64_t n_sitems = 0;
+  DevBuf<int2> split_info;    // per scratch slot: {first slot, nchunks}
+  DevBuf<int32_t> split_counter;
+  int64_t n_slots = 0;
+  DevBuf<float> scratch;      // n_slots × scratch_k
+  int64_t scratch_k = 0;
+  int32_t tile_cols = 64;
+  int32_t panel_rows = 64;
+  int64_t max_dense_per_panel = 0;
+};
+
+}  // namespace sr
+
+struct sr_csr_s {
+  int device = 0;
+  sr::HostCSR A;
+  bool reordered = false;
+  sr_reorder_params params{};
+  std::vector<int32_t> perm1, perm2;
+  sr::Tiling tiles;
+  sr_plan_stats stats{};
+  std::vector<int32_t> shard_rows;
+  std::vector<int64_t> shard_nnz_ids;
+  sr::DevPlan plan;
+  int32_t last_launches = 0;
+  cudaStream_t init_stream = nullptr;
+};
+
+namespace sr {
+// tiler.cpp
+void tile_rows(const HostCSR& A, const std::vector<int32_t>& perm, int32_t panel_rows,
+               int32_t dense_min, Tiling& t);
+void avgsim_positions(const Tiling& t, uint64_t* num, uint64_t* den);
+// cluster.cpp
+void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t npairs,
+                  const uint64_t* pairs, const uint32_t* inter, const uint32_t* uni,
+                  int32_t threshold_size, int32_t* perm);
+void partition_panels(int64_t npanels, const int64_t* w, int32_t G, int64_t* cuts);
+// lsh.cu : device LSH candidate generation + exact Jaccard (sorted J order).
+// Returns candidate pairs sorted by (J desc, pair asc) with their (inter, uni).
+int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int64_t nnz,
+                   const sr_reorder_params& p, cudaStream_t s, std::vector<uint64_t>& pairs_by_j,
+                   std::vector<uint32_t>& inter, std::vector<uint32_t>& uni, int64_t* E);
+// exec.cu : launchers
+int launch_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int64_t ldc,
+                cudaStream_t s, int32_t* launches);
+int launch_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t ldy, int64_t K,
+                 float* out, cudaStream_t s, int32_t* launches);
+}  // namespace sr

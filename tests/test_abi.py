@@ -1,0 +1,100 @@
+"""CPU-only checks of the C ABI: libsr.so loads and exports every symbol include/sr.h
+declares; argument validation; the host half of the pipeline (Alg 3 clustering, panel
+partition) is bit-exact against the oracle.  No GPU compute calls."""
+import ctypes as C
+import os
+import re
+
+import numpy as np
+import pytest
+
+from synth import generators as g
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def sr():
+    import paper_conf_ppopp_jiangha20_b200 as sr
+    if not os.path.exists(sr.LIB_PATH):
+        from paper_conf_ppopp_jiangha20_b200 import _build
+        _build.build()
+    sr.lib()
+    return sr
+
+
+def test_exports_every_declared_symbol(sr):
+    hdr = open(os.path.join(ROOT, "include", "sr.h")).read()
+    declared = set(re.findall(r"^\s*(?:int|void|const char\*)\s+(sr_\w+)\s*\(", hdr, re.M))
+    assert len(declared) >= 15
+    lib = C.CDLL(sr.LIB_PATH)
+    for name in declared:
+        assert hasattr(lib, name), name
+    assert declared == set(sr.EXPORTED)
+
+
+def test_struct_layouts_match_header(sr):
+    # sr_reorder_params: 4 int32, u64 seed (8-aligned), 10 int32 -> 64 bytes
+    assert C.sizeof(sr.ReorderParams) == 64
+    assert sr.ReorderParams.seed.offset == 16
+    p = sr.default_params()
+    assert (p.siglen, p.bsize, p.threshold_size, p.max_bucket, p.seed) == (128, 2, 256, 32, 4)
+    assert (p.panel_rows, p.dense_min, p.tile_cols, p.mode) == (64, 2, 64, sr.AUTO)
+    assert (p.skip_dense_num, p.skip_dense_den, p.skip_sim_num, p.skip_sim_den) == (1, 10, 1, 10)
+
+
+def test_create_validates_before_touching_a_device(sr):
+    A = g.fig1a()
+    bad = A.colidx.copy()
+    bad[0] = 99
+    with pytest.raises(sr.SRError) as e:
+        sr.SparseMatrix(6, 6, A.rowptr, bad, A.vals)
+    assert e.value.code == sr.SR_EINVAL
+    dup = A.colidx.copy()
+    dup[1] = 0
+    with pytest.raises(sr.SRError) as e:
+        sr.SparseMatrix(6, 6, A.rowptr, dup, A.vals)
+    assert e.value.code == sr.SR_EINVAL
+    rp = A.rowptr.copy()
+    rp[2] = 1  # decreasing
+    with pytest.raises(sr.SRError) as e:
+        sr.SparseMatrix(6, 6, rp, A.colidx, A.vals)
+    assert e.value.code == sr.SR_EINVAL
+
+
+def _sorted_pairs(E):
+    return np.sort(E)
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3, 4])
+def test_host_cluster_bit_exact_vs_oracle(sr, oracle, seed):
+    A = g.random_csr(400, 120, 0.04, seed, empty_frac=0.15)
+    E = oracle.candidates(A.rowptr, A.colidx, 32, 2, 4, 0)
+    for thr in (2, 5, 256):
+        ref = oracle.cluster(A.rowptr, A.colidx, E, thr)
+        got = sr.host_cluster(A.rowptr, A.colidx, E, thr)
+        np.testing.assert_array_equal(got, ref)
+        inter, uni = oracle.jaccard_pairs(A.rowptr, A.colidx, E)
+        got2 = sr.host_cluster(A.rowptr, A.colidx, E, thr, inter=inter, uni=uni)
+        np.testing.assert_array_equal(got2, ref)
+
+
+def test_host_cluster_fig6(sr):
+    A = g.fig1a()
+    from oracle import oracle as O
+    assert sr.host_cluster(A.rowptr, A.colidx, O.pack_pairs([(0, 4), (2, 4)]), 256).tolist() == [0, 2, 4, 1, 3, 5]
+
+
+def test_host_cluster_rejects_unsorted_pairs(sr):
+    A = g.fig1a()
+    with pytest.raises(sr.SRError):
+        sr.host_cluster(A.rowptr, A.colidx, np.array([(2 << 32) | 4, 4], np.uint64), 256)
+
+
+@pytest.mark.parametrize("G", [1, 2, 3, 8])
+def test_host_partition_matches_oracle(sr, oracle, G):
+    rng = np.random.default_rng(G)
+    for _ in range(25):
+        w = rng.integers(0, 1000, size=int(rng.integers(1, 300)))
+        w[rng.random(w.size) < 0.2] = 0
+        np.testing.assert_array_equal(sr.host_partition(w, G), oracle.partition(w, G))

@@ -1,0 +1,304 @@
+"""GPU parity: libsr (C ABI, sm_100a kernels) against the CPU oracle on the same seeded
+inputs.  Plan metadata must be bit-exact; fp32 outputs must satisfy the north_star bound
+|err| <= 1e-4·Σ_k|a_ik||b_kj| (SpMM) and |err| <= 1e-4·|a_ij|·Σ_k|x_ik||y_jk| (SDDMM)."""
+import numpy as np
+import pytest
+
+from synth import generators as g
+
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-4
+
+
+@pytest.fixture(scope="module")
+def env():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.fail("a CUDA device is required for -m gpu tests")
+    import paper_conf_ppopp_jiangha20_b200 as sr
+    sr.lib()
+    return sr, torch
+
+
+def _spmm_check(oracle, A, B, C_gpu, rows=None):
+    if rows is None:
+        ref, bound = oracle.spmm_rows(A, B, np.arange(A.nrows))
+        got = C_gpu
+    else:
+        ref, bound = oracle.spmm_rows(A, B, rows)
+        got = C_gpu[rows]
+    err = np.abs(got.astype(np.float64) - ref)
+    bad = err > TOL * bound + 1e-30
+    assert not bad.any(), f"{bad.sum()} entries out of tolerance; worst {err.max()}"
+
+
+def _sddmm_check(oracle, A, X, Y, out_gpu):
+    ref, bound = oracle.sddmm(A, X, Y)
+    err = np.abs(out_gpu.astype(np.float64) - ref)
+    bad = err > TOL * bound + 1e-30
+    assert not bad.any(), f"{bad.sum()} entries out of tolerance; worst {err.max()}"
+
+
+def _run(env, A, K, params=None, seed=3):
+    sr, torch = env
+    M = sr.SparseMatrix.from_csr(A)
+    if params is not None:
+        M.reorder(params)
+    B = g.dense(A.ncols, K, seed=seed)
+    X = g.dense(A.nrows, K, seed=seed, stream=1)
+    Y = g.dense(A.ncols, K, seed=seed, stream=2)
+    Bd, Xd, Yd = (torch.from_numpy(t).cuda() for t in (B, X, Y))
+    C = M.spmm(Bd)
+    out = M.sddmm(Xd, Yd)
+    torch.cuda.synchronize()
+    return M, B, X, Y, C.cpu().numpy(), out.cpu().numpy()
+
+
+# ------------------------------------------------------------------ identity plan
+@pytest.mark.parametrize("K", [32, 128])
+def test_tiny_identity_plan(env, oracle, K):
+    A = g.tiny()
+    M, B, X, Y, C, out = _run(env, A, K)
+    _spmm_check(oracle, A, B, C)
+    _sddmm_check(oracle, A, X, Y, out)
+    assert M.last_launch_count() >= 1
+
+
+# ------------------------------------------------------------------ plan bit-exactness
+def _plan_kw(panel_rows=8, mode=1, max_bucket=0, tile_cols=16):
+    return dict(siglen=128, bsize=2, seed=4, max_bucket=max_bucket, threshold_size=256,
+                panel_rows=panel_rows, dense_min=2, mode=mode)
+
+
+def _assert_plan_equal(M, ref):
+    np.testing.assert_array_equal(M.perm(1), ref["perm1"])
+    np.testing.assert_array_equal(M.perm(2), ref["perm2"])
+    t = M.tiles()
+    for k in ("dense_ptr", "dense_cols", "drow_ptr", "d_slot", "d_pos", "rrow_ptr", "r_col", "r_pos"):
+        np.testing.assert_array_equal(t[k], ref[k], err_msg=k)
+    st = M.stats()
+    for k in ("dense0", "dense1", "avgsim_num", "avgsim_den", "round1", "round2", "E1", "E2", "npanels",
+              "ndense_cols"):
+        assert st[k] == ref["stats"][k], k
+
+
+@pytest.mark.parametrize("mode", [0, 1, 2])
+@pytest.mark.parametrize("panel_rows,max_bucket", [(8, 0), (64, 0), (16, 4)])
+def test_tiny_plan_bit_exact(env, oracle, mode, panel_rows, max_bucket):
+    sr, _ = env
+    A = g.tiny()
+    kw = _plan_kw(panel_rows, mode, max_bucket)
+    ref = oracle.plan(A, **kw)
+    M = sr.SparseMatrix.from_csr(A)
+    M.reorder(sr.default_params(**kw, tile_cols=16))
+    _assert_plan_equal(M, ref)
+
+
+def test_worked_example_plan(env, oracle):
+    """Fig 1a in FORCE mode, panel 3, dense >= 2."""
+    sr, _ = env
+    A = g.fig1a()
+    kw = _plan_kw(3, 1, 0)
+    M = sr.SparseMatrix.from_csr(A)
+    M.reorder(sr.default_params(**kw, tile_cols=2))
+    _assert_plan_equal(M, oracle.plan(A, **kw))
+    # DenseRatio0 = 2/13
+    assert M.stats()["dense0"] == 2
+
+
+# ------------------------------------------------------------------ numerics over the plan
+@pytest.mark.parametrize("K", [1, 3, 4, 8, 32, 36, 64, 128, 132, 256])
+def test_k_sweep_forced_plan(env, oracle, K):
+    sr, _ = env
+    A = g.random_csr(700, 500, 0.03, 5, empty_frac=0.1)
+    M, B, X, Y, C, out = _run(env, A, K, sr.default_params(**_plan_kw(16, 1, 8), tile_cols=8))
+    assert M.stats()["dense1"] > 0
+    _spmm_check(oracle, A, B, C)
+    _sddmm_check(oracle, A, X, Y, out)
+
+
+@pytest.mark.parametrize("tile_cols", [1, 5, 64, 1024])
+def test_tile_widths(env, oracle, tile_cols):
+    sr, _ = env
+    A = g.random_csr(300, 60, 0.2, 9, empty_frac=0.05)  # dense-ish -> many dense columns
+    M, B, X, Y, C, out = _run(env, A, 32, sr.default_params(**_plan_kw(32, 1, 0), tile_cols=tile_cols))
+    assert M.stats()["ndense_cols"] > 60
+    _spmm_check(oracle, A, B, C)
+    _sddmm_check(oracle, A, X, Y, out)
+
+
+def test_long_rows_split_and_rmw(env, oracle):
+    """Rows far longer than one work item (split + ordered combine), some of them also
+    with dense-tile nnz (read-modify-write of C), and empty rows (zero fill)."""
+    sr, _ = env
+    rng = np.random.default_rng(0)
+    rows, cols = [], []
+    n, m = 200, 20000
+    for i in range(n):
+        d = 5000 if i % 37 == 0 else (0 if i % 11 == 0 else int(rng.integers(1, 40)))
+        c = rng.choice(m, size=d, replace=False)
+        rows.append(np.full(d, i))
+        cols.append(c)
+    # a shared hub block so panels get dense columns
+    hub = np.arange(32)
+    for i in range(0, n, 3):
+        rows.append(np.full(32, i))
+        cols.append(hub)
+    rowptr, colidx = g._from_coo(n, m, np.concatenate(rows), np.concatenate(cols))
+    A = g.CSR(n, m, rowptr, colidx, g._uniform_vals(colidx.size, 3))
+    for params in (None, sr.default_params(**_plan_kw(16, 1, 8)), sr.default_params(**_plan_kw(16, 2, 0))):
+        for K in (32, 128):
+            M, B, X, Y, C, out = _run(env, A, K, params)
+            _spmm_check(oracle, A, B, C)
+            _sddmm_check(oracle, A, X, Y, out)
+            # the result is deterministic (ordered combine of split rows)
+            _, _, _, _, C2, _ = _run(env, A, K, params)
+            np.testing.assert_array_equal(C, C2)
+
+
+def test_unsorted_input_keeps_caller_nnz_order(env, oracle):
+    sr, _ = env
+    A = g.random_csr(120, 90, 0.1, 12, empty_frac=0.1)
+    U = g.shuffle_within_rows(A, seed=3)
+    for params in (None, sr.default_params(**_plan_kw(8, 1, 0))):
+        M, B, X, Y, C, out = _run(env, U, 32, params)
+        _sddmm_check(oracle, U, X, Y, out)  # oracle works in the given (unsorted) order
+        _spmm_check(oracle, U, B, C)
+        if params is not None:
+            ref = oracle.plan(A, **_plan_kw(8, 1, 0))  # plan of the canonical matrix
+            np.testing.assert_array_equal(M.perm(1), ref["perm1"])
+            t = M.tiles()
+            # d_pos / r_pos refer to the caller's (unsorted) positions
+            np.testing.assert_array_equal(np.sort(np.concatenate([t["d_pos"], t["r_pos"]])), np.arange(U.nnz))
+            np.testing.assert_array_equal(U.colidx[t["r_pos"]], t["r_col"])
+
+
+def test_strided_and_misaligned_operands(env, oracle):
+    sr, torch = env
+    A = g.random_csr(150, 100, 0.08, 4, empty_frac=0.1)
+    M = sr.SparseMatrix.from_csr(A)
+    M.reorder(sr.default_params(**_plan_kw(16, 1, 0)))
+    K = 32
+    B = g.dense(100, K)
+    # ldb = 40 (vector path), and a 1-float offset base (scalar path)
+    Bbig = torch.zeros((100, 41), device="cuda")
+    Bbig[:, :K] = torch.from_numpy(B).cuda()
+    C1 = torch.full((150, 40), 7.0, device="cuda")
+    M.spmm(Bbig[:, :K], C1[:, :K])
+    Bmis = torch.zeros(100 * K + 1, device="cuda")
+    Bmis[1:] = torch.from_numpy(B.reshape(-1)).cuda()
+    C2 = M.spmm(Bmis[1:].view(100, K))
+    torch.cuda.synchronize()
+    _spmm_check(oracle, A, B, C1[:, :K].cpu().numpy())
+    _spmm_check(oracle, A, B, C2.cpu().numpy())
+    assert torch.all(C1[:, K:] == 7.0)  # padding columns untouched
+
+
+def test_empty_and_degenerate(env, oracle):
+    sr, torch = env
+    # all rows empty
+    A = g.CSR(10, 10, np.zeros(11, np.int64), np.zeros(0, np.int32), np.zeros(0, np.float32))
+    M = sr.SparseMatrix.from_csr(A)
+    C = M.spmm(torch.ones((10, 8), device="cuda"))
+    torch.cuda.synchronize()
+    assert torch.all(C == 0)
+    M.reorder(sr.default_params(**_plan_kw(4, 1, 0)))
+    C = M.spmm(torch.ones((10, 8), device="cuda"))
+    torch.cuda.synchronize()
+    assert torch.all(C == 0)
+    # single row / single column
+    for A in (g.random_csr(1, 64, 0.5, 1), g.random_csr(64, 1, 0.5, 2), g.diagonal(100)):
+        M, B, X, Y, C, out = _run(env, A, 8, sr.default_params(**_plan_kw(8, 1, 0)))
+        _spmm_check(oracle, A, B, C)
+        _sddmm_check(oracle, A, X, Y, out)
+
+
+def test_reorder_twice_is_a_state_error(env):
+    sr, _ = env
+    M = sr.SparseMatrix.from_csr(g.tiny())
+    M.reorder(sr.default_params())
+    with pytest.raises(sr.SRError) as e:
+        M.reorder(sr.default_params())
+    assert e.value.code == sr.SR_ESTATE
+
+
+def test_bad_params(env):
+    sr, _ = env
+    M = sr.SparseMatrix.from_csr(g.tiny())
+    for kw in (dict(siglen=10, bsize=3), dict(panel_rows=0), dict(tile_cols=0), dict(threshold_size=1),
+               dict(mode=7), dict(world=2, rank=2)):
+        with pytest.raises(sr.SRError) as e:
+            M.reorder(sr.default_params(**kw))
+        assert e.value.code == sr.SR_EINVAL, kw
+    with pytest.raises(sr.SRError) as e:
+        M.reorder(sr.default_params(siglen=12, bsize=4))
+    assert e.value.code == sr.SR_EUNSUPPORTED
+
+
+# ------------------------------------------------------------------ sharded plans on one GPU
+@pytest.mark.parametrize("world", [2, 3])
+def test_shard_simulation(env, oracle, world):
+    """Run every shard's plan on the same GPU and reassemble (SURVEY §4 tier 4a)."""
+    sr, torch = env
+    A = g.random_csr(500, 300, 0.03, 21, empty_frac=0.1)
+    K = 32
+    B = torch.from_numpy(g.dense(300, K)).cuda()
+    X = torch.from_numpy(g.dense(500, K, stream=1)).cuda()
+    Y = torch.from_numpy(g.dense(300, K, stream=2)).cuda()
+    C = np.full((500, K), np.nan, np.float32)
+    out = np.full(A.nnz, np.nan, np.float32)
+    ref_cuts = None
+    for r in range(world):
+        M = sr.SparseMatrix.from_csr(A)
+        M.reorder(sr.default_params(**_plan_kw(16, 1, 0), world=world, rank=r))
+        st = M.stats()
+        Cr = M.spmm(B)
+        outr = M.sddmm(X, Y)
+        torch.cuda.synchronize()
+        rows = M.shard_rows()
+        assert Cr.shape[0] == rows.size == st["shard_nrows"]
+        C[rows] = Cr.cpu().numpy()
+        out[M.shard_nnz_ids()] = outr.cpu().numpy()
+        if ref_cuts is None:
+            ref = oracle.plan(A, **_plan_kw(16, 1, 0))
+            P = 16
+            w = [int(ref["drow_ptr"][min(500, (p + 1) * P)] - ref["drow_ptr"][p * P]
+                     + ref["rrow_ptr"][min(500, (p + 1) * P)] - ref["rrow_ptr"][p * P]) for p in range(ref["npanels"])]
+            ref_cuts = oracle.partition(np.array(w), world)
+        assert (st["shard_panel_begin"], st["shard_panel_end"]) == (ref_cuts[r], ref_cuts[r + 1])
+    assert not np.isnan(C).any() and not np.isnan(out).any()
+    _spmm_check(oracle, A, B.cpu().numpy(), C)
+    _sddmm_check(oracle, A, X.cpu().numpy(), Y.cpu().numpy(), out)
+
+
+# ------------------------------------------------------------------ full-size configs
+@pytest.mark.slow
+def test_rmat_full_size_sampled(env, oracle):
+    """C2 at its full size in the launch configuration bench.py times (K=128 and 32):
+    plan bit-exact vs the oracle, outputs checked on 2000 sampled rows / all SDDMM nnz of
+    those rows."""
+    sr, torch = env
+    A = g.rmat()
+    kw = dict(siglen=128, bsize=2, seed=4, max_bucket=32, threshold_size=256, panel_rows=64, dense_min=2,
+              mode=0)
+    M = sr.SparseMatrix.from_csr(A)
+    M.reorder(sr.default_params(**kw))
+    ref = oracle.plan(A, **kw)
+    _assert_plan_equal(M, ref)
+    rng = np.random.default_rng(0)
+    deg = np.diff(A.rowptr)
+    rows = np.unique(np.concatenate([rng.integers(0, A.nrows, 2000), np.argsort(deg)[-20:]]))
+    for K in (128, 32):
+        B = g.dense(A.ncols, K)
+        C = M.spmm(torch.from_numpy(B).cuda())
+        torch.cuda.synchronize()
+        _spmm_check(oracle, A, B, C.cpu().numpy(), rows=rows)
+    X, Y = g.dense(A.nrows, 128, stream=1), g.dense(A.ncols, 128, stream=2)
+    out = M.sddmm(torch.from_numpy(X).cuda(), torch.from_numpy(Y).cuda()).cpu().numpy()
+    sel = np.concatenate([np.arange(A.rowptr[r], A.rowptr[r + 1]) for r in rows])
+    sub = g.CSR(rows.size, A.ncols, np.concatenate([[0], np.cumsum(deg[rows])]).astype(np.int64),
+                A.colidx[sel], A.vals[sel])
+    ref_o, bound = oracle.sddmm(sub, X[rows], Y)
+    err = np.abs(out[sel] - ref_o)
+    assert not (err > TOL * bound + 1e-30).any()
