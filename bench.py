@@ -1,0 +1,432 @@
+#!/usr/bin/env python3
+"""bench.py — SpMM / SDDMM throughput of the row-reordered, adaptively tiled path on B200.
+
+Metric (BASELINE.json): SpMM/SDDMM GFLOP/s (2·nnz·K per op) and HBM GB/s as a fraction of
+roofline.  Workload at N=1: C2, the R-MAT scale-20 matrix (configs[1]), K=128.
+
+One step = one pass of the execution hot path over the planned matrix: C := A·B (SpMM)
+and out := A ⊙ (X·Yᵀ) on A's pattern (SDDMM), both through the C ABI (libsr.so).  The
+reorder preprocessing (LSH on the GPU + Alg 3 on the host + ASpT tiling) runs once
+before the timed region and is reported separately (`preprocess`), as the paper does
+(P:277).  Inputs are resident in HBM; a 512 MB write flushes L2 between steps
+(outside the device-timed intervals).  Multi-GPU: torchrun, one rank per GPU, rank r
+computes its nnz-balanced panel shard (strong scaling, no collective in the step).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                  [--config rmat] [--K 128] [--ops spmm,sddmm]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from synth import generators as gen  # noqa: E402
+
+PAPER_CONTEXT = ("P100 (paper, P:334, P:350): ASpT-RR up to 2.91x SpMM vs best of ASpT-NR/cuSPARSE and "
+                 "up to 3.19x SDDMM vs ASpT-NR; geomean 1.19x / 1.49x (K=1024)")
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="rmat", choices=list(gen.CONFIGS))
+    ap.add_argument("--K", type=int, default=128)
+    ap.add_argument("--ops", default="spmm,sddmm")
+    ap.add_argument("--mode", default="auto", choices=["auto", "force", "off"])
+    ap.add_argument("--panel-rows", type=int, default=64)
+    ap.add_argument("--tile-cols", type=int, default=64)
+    ap.add_argument("--max-bucket", type=int, default=32)
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target CPU work of cpu_baseline")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--gather", action="store_true", help="also time the optional NCCL all-gather of C")
+    ap.add_argument("--min-warm-s", type=float, default=1.0, help="keep warming up until this long (clocks)")
+    return ap.parse_args()
+
+
+def measured_peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(path):
+        with open(path) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu: int):
+        self.gpu = gpu
+        self.proc = None
+        self.path = f"/tmp/bench_clocks_{os.getpid()}.csv"
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                                          "-lms", "100", "-i", str(self.gpu)], stdout=open(self.path, "w"),
+                                         stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self) -> dict:
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        self.proc.wait()
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in open(self.path):
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                smax.append(float(parts[2]))
+            except ValueError:
+                continue
+            for n, v in zip(names, parts[5:9]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        os.unlink(self.path)
+        load = [s for s in sm if s > 0.5 * max(sm)] if sm else []
+        return {"sm_mhz": statistics.median(load) if load else None, "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ----------------------------------------------------------------------------- oracle legs
+def oracle_sample(A, K, target_s, ops):
+    """Time the CPU oracle (oracle/, fp64, OpenMP over the host cores) on a bounded row
+    sample of the workload: rows [0, R) with R grown until ~target_s of work."""
+    from oracle import oracle as O
+    O.build()
+    B = gen.dense(A.ncols, K, stream=0)
+    Y = gen.dense(A.ncols, K, stream=2) if "sddmm" in ops else None
+    R = max(1, A.nrows // 256)
+    while True:
+        sub = gen.CSR(R, A.ncols, A.rowptr[:R + 1].copy(), A.colidx[:A.rowptr[R]], A.vals[:A.rowptr[R]])
+        X = gen.dense(R, K, stream=1) if "sddmm" in ops else None
+        t0 = time.perf_counter()
+        if "spmm" in ops:
+            O.spmm(sub, B)
+        if "sddmm" in ops:
+            O.sddmm(sub, X, Y)
+        dt = time.perf_counter() - t0
+        if dt * 4 >= target_s or R >= A.nrows:
+            break
+        R = min(A.nrows, int(R * max(2.0, min(8.0, target_s / 2 / max(dt, 1e-3)))))
+    nnz = int(sub.rowptr[-1])
+    flops = 2.0 * nnz * K * len(ops)
+    return dict(sub=sub, B=B, X=X, Y=Y, rows=R, nnz=nnz, flops=flops, seconds=dt, O=O)
+
+
+def cpu_baseline(A, K, args, ops, name):
+    s = oracle_sample(A, K, args.cpu_seconds, ops)
+    # measured leg: ~target seconds of repeated passes over the sample
+    reps = max(1, int(round(args.cpu_seconds / max(s["seconds"], 1e-3))))
+    O = s["O"]
+    t0 = time.perf_counter()
+    for _ in range(reps):
+        if "spmm" in ops:
+            O.spmm(s["sub"], s["B"])
+        if "sddmm" in ops:
+            O.sddmm(s["sub"], s["X"], s["Y"])
+    dt = time.perf_counter() - t0
+    return {"value": s["flops"] * reps / dt / 1e9, "unit": "GFLOP/s", "cores": O.num_threads(), "kind": "oracle",
+            "sample": f"{name} rows [0,{s['rows']}) = {s['nnz']} nnz of {A.nnz}, K={K}, {'+'.join(ops)} in fp64, "
+                      f"{reps} pass(es), {dt:.1f} s"}
+
+
+def run_reference(args, A, ops, rank, world):
+    if rank != 0:
+        return
+    s = oracle_sample(A, args.K, max(2.0, args.cpu_seconds / 4), ops)
+    O = s["O"]
+
+    def step():
+        if "spmm" in ops:
+            O.spmm(s["sub"], s["B"])
+        if "sddmm" in ops:
+            O.sddmm(s["sub"], s["X"], s["Y"])
+    for _ in range(args.warmup):
+        step()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        step()
+    dt = time.perf_counter() - t0
+    value = s["flops"] * args.steps / dt / 1e9
+    line = {
+        "impl": "reference", "metric": "SpMM+SDDMM GFLOP/s (2*nnz*K per op)", "value": value, "unit": "GFLOP/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": args.config, "K": args.K, "ops": ops, "nnz": A.nnz, "nrows": A.nrows,
+                   "ncols": A.ncols},
+        "cpu_baseline": {"value": value, "unit": "GFLOP/s", "cores": O.num_threads(), "kind": "oracle",
+                         "sample": f"rows [0,{s['rows']}) = {s['nnz']} nnz of {A.nnz} per step"},
+        "e2e": {"value": value, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------------------- our arm
+def algorithmic_bytes(kind: str, tm: dict, K: int) -> float:
+    """Compulsory bytes of one launch: every sparse entry's (col, val) once,
+    every distinct gathered dense row once, every output written once."""
+    row = 4.0 * K
+    if kind == "spmm_sparse_rows":
+        return (8.0 * tm["sparse_nnz"] + 16.0 * tm["sparse_items"] + row * tm["sparse_distinct_cols"]
+                + row * (tm["sparse_rows"] + tm["zero_rows"]) + row * tm["rmw_rows"])
+    if kind == "spmm_dense_tiles":
+        return 8.0 * tm["dense_nnz"] + row * tm["dense_distinct_cols"] + row * tm["dense_rows"]
+    if kind == "sddmm_sparse_rows":
+        return (12.0 * tm["sparse_nnz"] + 16.0 * tm["sparse_items"] + row * tm["sparse_distinct_cols"]
+                + row * tm["sparse_rows"])
+    if kind == "sddmm_dense_tiles":
+        return 12.0 * tm["dense_nnz"] + row * tm["dense_distinct_cols"] + row * tm["dense_rows"]
+    raise KeyError(kind)
+
+
+def model_bytes(kind: str, tm: dict, K: int) -> float:
+    """SURVEY §8(d) bytes model: B-row traffic from the access-count model (O14)."""
+    row = 4.0 * K
+    if kind.endswith("sparse_rows"):
+        return algorithmic_bytes(kind, tm, K) + row * (tm["sparse_group_loads"] - tm["sparse_distinct_cols"])
+    return algorithmic_bytes(kind, tm, K) + row * (tm["dense_col_loads"] - tm["dense_distinct_cols"])
+
+
+def run_ours(args, A, ops, rank, world, local_rank):
+    import torch
+    import paper_conf_ppopp_jiangha20_b200 as sr
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    K = args.K
+    mode = {"auto": sr.AUTO, "force": sr.FORCE, "off": sr.OFF}[args.mode]
+    params = sr.default_params(mode=mode, panel_rows=args.panel_rows, tile_cols=args.tile_cols,
+                               max_bucket=args.max_bucket, world=world, rank=rank)
+    M = sr.SparseMatrix.from_csr(A, device=local_rank)
+    t0 = time.perf_counter()
+    st = M.reorder(params)
+    t_pre = time.perf_counter() - t0
+    tm = M.traffic_model()
+    B = torch.from_numpy(gen.dense(A.ncols, K, stream=0)).to(dev)
+    X = torch.from_numpy(gen.dense(A.nrows, K, stream=1)).to(dev)
+    Y = torch.from_numpy(gen.dense(A.ncols, K, stream=2)).to(dev)
+    C = torch.empty((M.out_rows, K), dtype=torch.float32, device=dev)
+    out = torch.empty(M.out_nnz, dtype=torch.float32, device=dev)
+    flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+    stream = torch.cuda.current_stream()
+    M.set_profiling(True)
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in ops]
+    kern_ms: dict = {}
+    launches = 0
+
+    def step(record: bool):
+        nonlocal launches
+        flush.fill_(1.0)
+        total = 0.0
+        for i, op in enumerate(ops):
+            ev[i][0].record(stream)
+            if op == "spmm":
+                M.spmm(B, C, stream=stream)
+            else:
+                M.sddmm(X, Y, out, stream=stream)
+            ev[i][1].record(stream)
+            n = M.last_launch_count()
+            times = M.last_kernel_times()  # waits for this op
+            total += ev[i][0].elapsed_time(ev[i][1])
+            if record:
+                launches += n
+                for name, ms in times:
+                    kern_ms.setdefault(name, []).append(ms)
+        return total
+
+    dist = world > 1
+    if dist:
+        import torch.distributed as tdist
+    clocks = ClockSampler(local_rank)
+    clocks.start()
+    t_w = time.perf_counter()
+    for i in range(max(3, args.warmup)):
+        step(False)
+    while time.perf_counter() - t_w < args.min_warm_s:  # let the sampler see the GPU under load
+        step(False)
+    if dist:
+        tdist.barrier()
+    torch.cuda.synchronize()
+    wall0 = time.perf_counter()
+    dev_ms = 0.0
+    for i in range(args.steps):
+        dev_ms += step(True)
+    torch.cuda.synchronize()
+    if dist:
+        tdist.barrier()
+    wall = time.perf_counter() - wall0
+    clk = clocks.stop()
+    t = torch.tensor([dev_ms], dtype=torch.float64, device=dev)
+    if dist:
+        tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
+    max_ms = float(t.item())
+    flops_per_step = 2.0 * A.nnz * K * len(ops)  # whole matrix, all ranks together
+    value = flops_per_step * args.steps / (max_ms / 1e3) / 1e9
+
+    # per-kernel roofline of the dominant kernel
+    peak, peak_src = measured_peaks()
+    kern = {k: {"launches": len(v), "avg_ms": sum(v) / len(v), "total_ms": sum(v)} for k, v in kern_ms.items()}
+    for k, d in kern.items():
+        d["algorithmic_bytes"] = algorithmic_bytes(k, tm, K)
+        d["model_bytes"] = model_bytes(k, tm, K)
+        d["achieved_gbs"] = d["algorithmic_bytes"] / (d["avg_ms"] / 1e3) / 1e9
+        d["model_gbs"] = d["model_bytes"] / (d["avg_ms"] / 1e3) / 1e9
+        d["share_of_step"] = d["total_ms"] / dev_ms if dev_ms > 0 else None
+    dom = max(kern, key=lambda k: kern[k]["total_ms"]) if kern else None
+    traffic = None
+    prof_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if dom and os.path.exists(prof_path):
+        with open(prof_path) as f:
+            tr = json.load(f)
+        key = f"{args.config}_K{K}_{dom}"
+        traffic = tr.get(key)
+    roofline = None
+    if dom:
+        d = kern[dom]
+        roofline = {"kernel": dom, "bound": "hbm", "achieved": d["achieved_gbs"], "peak": peak, "unit": "GB/s",
+                    "frac": d["achieved_gbs"] / peak, "traffic": traffic, "peak_source": peak_src,
+                    "algorithmic_bytes_per_launch": d["algorithmic_bytes"], "avg_ms": d["avg_ms"]}
+
+    # end to end through the public API with host buffers (pinned), per step
+    e2e = None
+    if args.e2e_steps > 0:
+        hB = torch.from_numpy(gen.dense(A.ncols, K, stream=0)).pin_memory()
+        hX = torch.from_numpy(gen.dense(A.nrows, K, stream=1)).pin_memory()
+        hY = hB if "sddmm" not in ops else torch.from_numpy(gen.dense(A.ncols, K, stream=2)).pin_memory()
+        hC = torch.empty(C.shape, dtype=torch.float32).pin_memory()
+        hO = torch.empty(out.shape, dtype=torch.float32).pin_memory()
+        h2d = (hB.numel() * 4 if "spmm" in ops else 0) + ((hX.numel() + hY.numel()) * 4 if "sddmm" in ops else 0)
+        d2h = (hC.numel() * 4 if "spmm" in ops else 0) + (hO.numel() * 4 if "sddmm" in ops else 0)
+        M.set_profiling(False)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        tot = 0.0
+        for i in range(args.e2e_steps + 1):
+            flush.fill_(1.0)
+            e0.record(stream)
+            if "spmm" in ops:
+                B.copy_(hB, non_blocking=True)
+                M.spmm(B, C, stream=stream)
+                hC.copy_(C, non_blocking=True)
+            if "sddmm" in ops:
+                X.copy_(hX, non_blocking=True)
+                Y.copy_(hY, non_blocking=True)
+                M.sddmm(X, Y, out, stream=stream)
+                hO.copy_(out, non_blocking=True)
+            e1.record(stream)
+            e1.synchronize()
+            if i > 0:
+                tot += e0.elapsed_time(e1)
+        te = torch.tensor([tot], dtype=torch.float64, device=dev)
+        if dist:
+            tdist.all_reduce(te, op=tdist.ReduceOp.MAX)
+        e2e = {"value": flops_per_step * args.e2e_steps / (float(te.item()) / 1e3) / 1e9, "unit": "GFLOP/s",
+               "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+               "note": "pinned host operands copied in and outputs copied out every step, through SparseMatrix"}
+
+    gather = None
+    if args.gather and dist and "spmm" in ops:
+        rows_max = torch.tensor([C.shape[0]], device=dev)
+        tdist.all_reduce(rows_max, op=tdist.ReduceOp.MAX)
+        pad = torch.zeros((int(rows_max.item()), K), device=dev)
+        pad[:C.shape[0]] = C
+        bufs = torch.empty((world, int(rows_max.item()), K), device=dev)
+        g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        g0.record()
+        tdist.all_gather_into_tensor(bufs, pad)
+        g1.record()
+        torch.cuda.synchronize()
+        gather = {"ms": g0.elapsed_time(g1), "bytes_per_rank": pad.numel() * 4}
+
+    if rank == 0:
+        cpu = None
+        if not args.no_cpu_baseline and world == 1:
+            cpu = cpu_baseline(A, K, args, ops, args.config)
+        stp = M.stats()
+        line = {
+            "metric": "SpMM+SDDMM GFLOP/s (2*nnz*K per op) and HBM GB/s (fraction of roofline)",
+            "value": value, "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": max_ms / args.steps, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"{args.config} (configs[{list(gen.CONFIGS).index(args.config)}])",
+                       "nrows": A.nrows, "ncols": A.ncols, "nnz": A.nnz, "K": K, "ops": ops,
+                       "parallelism": f"row-panel shards x{world}" if world > 1 else "single GPU",
+                       "l2": "512 MB write between steps (outside timed intervals); B/X/Y > L2",
+                       "plan": {"mode": args.mode, "panel_rows": args.panel_rows, "tile_cols": args.tile_cols,
+                                "max_bucket": args.max_bucket, "siglen": 128, "bsize": 2, "threshold_size": 256,
+                                "seed": 4}},
+            "roofline": roofline,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": launches,
+            "clocks": clk,
+            "kernels": kern,
+            "per_op_gflops": None,
+            "preprocess": {"seconds": t_pre, "lsh1_s": stp["t_lsh1_s"], "cluster1_s": stp["t_cluster1_s"],
+                           "tile_s": stp["t_tile_s"], "lsh2_s": stp["t_lsh2_s"], "cluster2_s": stp["t_cluster2_s"],
+                           "round1": stp["round1"], "round2": stp["round2"], "E1": stp["E1"], "E2": stp["E2"],
+                           "dense_ratio0": stp["dense0"] / max(1, stp["nnz"]),
+                           "dense_ratio": stp["dense1"] / max(1, stp["nnz"]),
+                           "avgsim": (stp["avgsim_num"] / stp["avgsim_den"]) if stp["avgsim_den"] else 0.0,
+                           "ratio_to_step": t_pre / (max_ms / args.steps / 1e3)},
+            "traffic_model": tm,
+            "wall_s": wall,
+            "gather": gather,
+            "paper_context": PAPER_CONTEXT,
+        }
+        per_op = {}
+        for name in ("spmm", "sddmm"):
+            ks = [k for k in kern if k.startswith(name)]
+            if ks:
+                ms = sum(kern[k]["avg_ms"] for k in ks)
+                per_op[name] = {"ms": ms, "gflops": 2.0 * A.nnz * K / (ms / 1e3) / 1e9 if world == 1 else None}
+        line["per_op_gflops"] = per_op
+        print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    ops = [o.strip() for o in args.ops.split(",") if o.strip()]
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference" and rank != 0:
+        return  # the oracle arm runs on rank 0 only
+    A = gen.make(args.config)
+    if args.impl == "reference":
+        run_reference(args, A, ops, rank, world)
+        return
+    if world > 1:
+        import torch
+        import torch.distributed as tdist
+        torch.cuda.set_device(local_rank)
+        tdist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    run_ours(args, A, ops, rank, world, local_rank)
+    if world > 1:
+        import torch.distributed as tdist
+        tdist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -166,6 +166,33 @@ int sr_shard_nnz_ids(sr_csr h, int64_t* ids_out, int64_t cap, int64_t* len);
 /* Kernel launches the last sr_spmm / sr_sddmm call issued on this handle. */
 int sr_last_launch_count(sr_csr h, int32_t* n);
 
+/* ---------------------------------------------------------------------------
+ * Measurement hooks (bench.py): the bytes model of the current plan and per-launch
+ * device times of the last sr_spmm / sr_sddmm call.
+ * -------------------------------------------------------------------------*/
+typedef struct {
+  int64_t dense_nnz, sparse_nnz;        /* nnz served by phase D (tiles) / phase S (remainder) */
+  int64_t dense_panels, sparse_items;   /* CTAs of phase D; warps (work items) of phase S      */
+  int64_t dense_rows;                   /* rows written by phase D                             */
+  int64_t sparse_rows;                  /* remainder rows (phase S writes or read-modify-writes) */
+  int64_t zero_rows;                    /* rows with no nnz (phase S zero-fills them)          */
+  int64_t rmw_rows;                     /* rows with both dense-tile and remainder nnz         */
+  int64_t dense_col_loads;              /* Σ_p |D_p|: B/Y rows staged into shared memory */
+  int64_t dense_distinct_cols;          /* distinct columns over all D_p                       */
+  int64_t sparse_group_loads;           /* access model O14 of phase S (8 warps per CTA) */
+  int64_t sparse_distinct_cols;         /* distinct columns of the remainder                   */
+} sr_traffic_model;
+
+int sr_get_traffic_model(sr_csr h, sr_traffic_model* out);
+
+/* enable != 0: every later sr_spmm / sr_sddmm records a CUDA event pair around each of its
+ * kernel launches on the call's stream. */
+int sr_set_profiling(sr_csr h, int enable);
+
+/* Device time of each launch of the last sr_spmm / sr_sddmm call (waits for its events).
+ * kinds: 1 = spmm phase D, 2 = spmm phase S, 3 = sddmm phase D, 4 = sddmm phase S. */
+int sr_last_kernel_times(sr_csr h, int32_t* kinds, float* ms, int32_t cap, int32_t* n);
+
 const char* sr_last_error(void);
 
 /* ---------------------------------------------------------------------------

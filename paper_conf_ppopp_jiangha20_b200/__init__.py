@@ -49,9 +49,21 @@ class PlanStats(C.Structure):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
 
+class TrafficModel(C.Structure):
+    _fields_ = [(k, C.c_int64) for k in (
+        "dense_nnz", "sparse_nnz", "dense_panels", "sparse_items", "dense_rows", "sparse_rows", "zero_rows",
+        "rmw_rows", "dense_col_loads", "dense_distinct_cols", "sparse_group_loads", "sparse_distinct_cols")]
+
+    def as_dict(self) -> dict:
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+KERNEL_KINDS = {1: "spmm_dense_tiles", 2: "spmm_sparse_rows", 3: "sddmm_dense_tiles", 4: "sddmm_sparse_rows"}
+
 EXPORTED = ("sr_csr_create", "sr_default_params", "sr_reorder", "sr_spmm", "sr_sddmm", "sr_destroy",
             "sr_get_perm", "sr_get_plan_stats", "sr_export_tiles", "sr_shard_rows", "sr_shard_nnz_ids",
-            "sr_last_launch_count", "sr_last_error", "sr_host_cluster", "sr_host_partition", "sr_version")
+            "sr_last_launch_count", "sr_last_error", "sr_host_cluster", "sr_host_partition", "sr_version",
+            "sr_get_traffic_model", "sr_set_profiling", "sr_last_kernel_times")
 
 _lib = None
 
@@ -82,6 +94,9 @@ def lib():
         "sr_host_cluster": (C.c_int, [i64, P, P, i64, P, P, P, i32, P]),
         "sr_host_partition": (C.c_int, [i64, P, i32, P]),
         "sr_version": (C.c_char_p, []),
+        "sr_get_traffic_model": (C.c_int, [P, C.POINTER(TrafficModel)]),
+        "sr_set_profiling": (C.c_int, [P, C.c_int]),
+        "sr_last_kernel_times": (C.c_int, [P, P, P, i32, C.POINTER(i32)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -205,6 +220,23 @@ class SparseMatrix:
         out = np.empty(n.value, np.int64)
         _check(lib().sr_shard_nnz_ids(self._h, out.ctypes.data_as(C.c_void_p), out.size, C.byref(n)))
         return out
+
+    def traffic_model(self) -> dict:
+        t = TrafficModel()
+        _check(lib().sr_get_traffic_model(self._h, C.byref(t)))
+        return t.as_dict()
+
+    def set_profiling(self, on: bool = True):
+        _check(lib().sr_set_profiling(self._h, 1 if on else 0))
+
+    def last_kernel_times(self) -> list:
+        """[(kernel name, device ms), ...] of the last spmm / sddmm call (waits for it)."""
+        kinds = (C.c_int32 * 4)()
+        ms = (C.c_float * 4)()
+        n = C.c_int32()
+        _check(lib().sr_last_kernel_times(self._h, C.cast(kinds, C.c_void_p), C.cast(ms, C.c_void_p), 4,
+                                          C.byref(n)))
+        return [(KERNEL_KINDS[kinds[i]], float(ms[i])) for i in range(n.value)]
 
     def last_launch_count(self) -> int:
         n = C.c_int32()

@@ -69,6 +69,39 @@ struct ItemBuilder {
   }
 };
 
+// Bytes model of phase S: entries of consecutive groups of 8 items (one CTA) that share a
+// column load it once (access model O14 / P:111); distinct columns = compulsory.
+void sparse_traffic(const ItemBuilder& ib, int64_t n_nonzero, int64_t n_zero, const std::vector<int2>& ent,
+                    int64_t N, sr_traffic_model& t) {
+  std::vector<int64_t> mark((size_t)N, -1);
+  std::vector<uint8_t> seen((size_t)N, 0);
+  int64_t loads = 0, distinct = 0, nnz = 0, rows = 0;
+  for (int64_t it = 0; it < n_nonzero; ++it) {
+    const int64_t grp = it / 8;
+    const Item& x = ib.items[it];
+    nnz += x.e1 - x.e0;
+    const uint32_t m = ib.meta[it];
+    if (!(m & kItemSplit) || (m & kItemSlotMask) == (uint32_t)ib.split_info[m & kItemSlotMask].x) ++rows;
+    for (int32_t e = x.e0; e < x.e1; ++e) {
+      const int32_t c = ent[e].x;
+      if (mark[c] != grp) {
+        mark[c] = grp;
+        ++loads;
+      }
+      if (!seen[c]) {
+        seen[c] = 1;
+        ++distinct;
+      }
+    }
+  }
+  t.sparse_nnz = nnz;
+  t.sparse_items = n_nonzero + n_zero;
+  t.sparse_rows = rows;
+  t.zero_rows = n_zero;
+  t.sparse_group_loads = loads;
+  t.sparse_distinct_cols = distinct;
+}
+
 int upload_items(DevPlan& P, ItemBuilder& ib, int64_t n_sddmm_items, cudaStream_t s) {
   P.n_items = (int64_t)ib.items.size();
   P.n_sitems = n_sddmm_items;
@@ -117,6 +150,8 @@ int build_identity_plan(sr_csr_s* h, cudaStream_t s) {
     ib.items.push_back(Item{0, 0, r, r});
     ib.meta.push_back(0u);
   }
+  std::memset(&P.traffic, 0, sizeof(P.traffic));
+  sparse_traffic(ib, n_nonzero, (int64_t)zero_rows.size(), ent, A.N, P.traffic);
   SR_TRY(upload_items(P, ib, n_nonzero, s));
   P.n_dpanels = 0;
   SR_CUDA_TRY(cudaStreamSynchronize(s));
@@ -213,6 +248,28 @@ int build_exec_plan(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s) {
       const int32_t out = sharded ? (int32_t)(q - q0s) : perm1[q];
       ib.items.push_back(Item{0, 0, perm1[q], out});
       ib.meta.push_back(0u);
+    }
+  }
+  // bytes model
+  sr_traffic_model& tm = P.traffic;
+  std::memset(&tm, 0, sizeof(tm));
+  sparse_traffic(ib, n_nonzero, (int64_t)ib.items.size() - n_nonzero, se, A.N, tm);
+  {
+    std::vector<uint8_t> seen((size_t)A.N, 0);
+    for (const DPanel& d : dp) {
+      tm.dense_col_loads += d.dc1 - d.dc0;
+      for (int32_t k = d.dc0; k < d.dc1; ++k)
+        if (!seen[T.dense_cols[k]]) {
+          seen[T.dense_cols[k]] = 1;
+          ++tm.dense_distinct_cols;
+        }
+    }
+    tm.dense_panels = (int64_t)dp.size();
+    for (int64_t q = q0s; q < q1s; ++q) {
+      const bool d = T.drow_ptr[q + 1] > T.drow_ptr[q], r = T.rrow_ptr[q + 1] > T.rrow_ptr[q];
+      tm.dense_nnz += T.drow_ptr[q + 1] - T.drow_ptr[q];
+      tm.dense_rows += d;
+      tm.rmw_rows += d && r;
     }
   }
   SR_TRY(P.s_ent.upload(se, s));
@@ -490,6 +547,8 @@ int sr_destroy(sr_csr h) {
     DeviceGuard dg(h->device);
     cudaDeviceSynchronize();
     if (h->init_stream) cudaStreamDestroy(h->init_stream);
+    for (cudaEvent_t e : h->plan.ev)
+      if (e) cudaEventDestroy(e);
     delete h;
   }
   return SR_OK;
@@ -557,6 +616,34 @@ int sr_shard_nnz_ids(sr_csr h, int64_t* ids_out, int64_t cap, int64_t* len) {
   *len = (int64_t)h->shard_nnz_ids.size();
   if (cap < *len) return ids_out ? einval("sr_shard_nnz_ids: capacity too small") : SR_OK;
   if (ids_out && *len) std::memcpy(ids_out, h->shard_nnz_ids.data(), *len * sizeof(int64_t));
+  return SR_OK;
+}
+
+int sr_get_traffic_model(sr_csr h, sr_traffic_model* out) {
+  if (!h || !out) return einval("sr_get_traffic_model: NULL argument");
+  *out = h->plan.traffic;
+  return SR_OK;
+}
+
+int sr_set_profiling(sr_csr h, int enable) {
+  if (!h) return einval("sr_set_profiling: NULL handle");
+  h->plan.profiling = enable != 0;
+  return SR_OK;
+}
+
+int sr_last_kernel_times(sr_csr h, int32_t* kinds, float* ms, int32_t cap, int32_t* n) {
+  if (!h || !n) return einval("sr_last_kernel_times: NULL argument");
+  DevPlan& P = h->plan;
+  *n = P.nrec;
+  if (cap < P.nrec) return (kinds || ms) ? einval("sr_last_kernel_times: capacity too small") : SR_OK;
+  DeviceGuard dg(h->device);
+  for (int32_t i = 0; i < P.nrec; ++i) {
+    SR_CUDA_TRY(cudaEventSynchronize(P.ev[2 * i + 1]));
+    float t = 0.f;
+    SR_CUDA_TRY(cudaEventElapsedTime(&t, P.ev[2 * i], P.ev[2 * i + 1]));
+    if (kinds) kinds[i] = P.kinds[i];
+    if (ms) ms[i] = t;
+  }
   return SR_OK;
 }
 

@@ -491,12 +491,14 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
       SR_CUDA_TRY(cudaGetLastError());
       return SR_OK;
     };
+    if (P.profiling) SR_TRY(prof_begin(P, 1, s));
     if (VEC == 4) {
       if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 8, true>));
       else SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 16, true>));
     } else {
       SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 16, false>));
     }
+    if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;
   }
   if (P.n_items > 0) {
@@ -505,10 +507,12 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
       P.scratch_k = K;
     }
     const unsigned grid = (unsigned)((P.n_items + kSparseWarps - 1) / kSparseWarps);
+    if (P.profiling) SR_TRY(prof_begin(P, 2, s));
     spmm_sparse_kernel<LPG, VEC, U><<<grid, kSparseWarps * 32, 0, s>>>(
         P.items.p, P.item_meta.p, P.n_items, P.s_ent.p, B, ldb, C, ldc, (int)K, P.scratch.p,
         P.split_info.p, P.split_counter.p);
     SR_CUDA_TRY(cudaGetLastError());
+    if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;
   }
   return SR_OK;
@@ -532,19 +536,23 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
       SR_CUDA_TRY(cudaGetLastError());
       return SR_OK;
     };
+    if (P.profiling) SR_TRY(prof_begin(P, 3, s));
     if (VEC == 4) {
       if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, U, NCH, 8, true>));
       else SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, U, NCH, 16, true>));
     } else {
       SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, U, NCH, 16, false>));
     }
+    if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;
   }
   if (P.n_sitems > 0) {
     const unsigned grid = (unsigned)((P.n_sitems + kSparseWarps - 1) / kSparseWarps);
+    if (P.profiling) SR_TRY(prof_begin(P, 4, s));
     sddmm_sparse_kernel<LPG, VEC, U, NCH><<<grid, kSparseWarps * 32, 0, s>>>(
         P.items.p, P.n_sitems, P.s_ent.p, P.s_oidx.p, X, ldx, Y, ldy, (int)K, out);
     SR_CUDA_TRY(cudaGetLastError());
+    if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;
   }
   return SR_OK;
@@ -552,9 +560,26 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
 
 }  // namespace
 
+int prof_begin(DevPlan& P, int kind, cudaStream_t s) {
+  if (P.nrec >= 4) return SR_OK;
+  for (int i = 0; i < 8; ++i)
+    if (!P.ev[i]) SR_CUDA_TRY(cudaEventCreate(&P.ev[i]));
+  P.kinds[P.nrec] = kind;
+  SR_CUDA_TRY(cudaEventRecord(P.ev[2 * P.nrec], s));
+  return SR_OK;
+}
+
+int prof_end(DevPlan& P, cudaStream_t s) {
+  if (P.nrec >= 4) return SR_OK;
+  SR_CUDA_TRY(cudaEventRecord(P.ev[2 * P.nrec + 1], s));
+  ++P.nrec;
+  return SR_OK;
+}
+
 int launch_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int64_t ldc,
                 cudaStream_t s, int32_t* launches) {
   *launches = 0;
+  h->plan.nrec = 0;
   const bool vec = (K % 4 == 0) && (ldb % 4 == 0) && (ldc % 4 == 0) &&
                    ((uintptr_t)B % 16 == 0) && ((uintptr_t)C % 16 == 0);
   const int VEC = vec ? 4 : 1;
@@ -571,6 +596,7 @@ int launch_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, i
 int launch_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t ldy, int64_t K,
                  float* out, cudaStream_t s, int32_t* launches) {
   *launches = 0;
+  h->plan.nrec = 0;
   const bool vec = (K % 4 == 0) && (ldx % 4 == 0) && (ldy % 4 == 0) &&
                    ((uintptr_t)X % 16 == 0) && ((uintptr_t)Y % 16 == 0);
   const int VEC = vec ? 4 : 1;

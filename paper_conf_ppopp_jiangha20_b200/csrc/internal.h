@@ -136,7 +136,17 @@ struct DevPlan {
   int32_t tile_cols = 64;
   int32_t panel_rows = 64;
   int64_t max_dense_per_panel = 0;
+  sr_traffic_model traffic{};
+  // profiling (sr_set_profiling)
+  bool profiling = false;
+  cudaEvent_t ev[8] = {};
+  int32_t kinds[4] = {};
+  int32_t nrec = 0;
 };
+
+// profiling helpers (exec.cu)
+int prof_begin(DevPlan& P, int kind, cudaStream_t s);
+int prof_end(DevPlan& P, cudaStream_t s);
 
 }  // namespace sr
 
