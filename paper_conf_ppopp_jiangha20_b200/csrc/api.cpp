@@ -153,7 +153,7 @@ int build_identity_plan(sr_csr_s* h, cudaStream_t s) {
   std::memset(&P.traffic, 0, sizeof(P.traffic));
   sparse_traffic(ib, n_nonzero, (int64_t)zero_rows.size(), ent, A.N, P.traffic);
   SR_TRY(upload_items(P, ib, n_nonzero, s));
-  P.n_dpanels = 0;
+  P.n_units = 0;
   SR_CUDA_TRY(cudaStreamSynchronize(s));
   return SR_OK;
 }
@@ -189,34 +189,84 @@ int build_exec_plan(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s) {
       }
     }
   }
-  // phase D
-  std::vector<DPanel> dp;
-  int64_t maxd = 0;
+  // phase D: tiles of tile_cols dense columns, tile-major entries, units of <= kMaxUnitTiles tiles
+  // execution tile width: the plan's tiles (tile_cols, reported in the metadata) are staged
+  // in sub-tiles of at most kMaxExecTile columns so two stages of K<=128 fit in 64 KB
+  const int32_t TW = std::min(h->params.tile_cols, kMaxExecTile);
+  std::vector<DUnit> units;
+  std::vector<int2> dsplit;
+  std::vector<int32_t> trp;
+  std::vector<int2> de;
+  std::vector<int32_t> deo;
+  de.reserve((size_t)T.n_dense());
+  deo.reserve((size_t)T.n_dense());
+  int64_t maxd = 0, ntiles_total = 0, n_dslots = 0;
+  std::vector<int64_t> cur((size_t)PR);
   for (int64_t p = pb; p < pe; ++p) {
     const int64_t dc0 = T.dense_ptr[p], dc1 = T.dense_ptr[p + 1];
     if (dc1 == dc0) continue;
     const int64_t q0 = p * PR, nrows = std::min<int64_t>(M, q0 + PR) - q0;
-    dp.push_back(DPanel{(int32_t)q0, (int32_t)nrows, (int32_t)dc0, (int32_t)dc1});
-    maxd = std::max(maxd, dc1 - dc0);
+    const int64_t nd = dc1 - dc0, nt = (nd + TW - 1) / TW;
+    maxd = std::max(maxd, nd);
+    for (int64_t r = 0; r < nrows; ++r) cur[r] = T.drow_ptr[q0 + r];
+    const int64_t tile_base = ntiles_total;
+    for (int64_t t = 0; t < nt; ++t) {
+      const int64_t s_hi = (t + 1) * TW;
+      for (int64_t r = 0; r < PR; ++r) {
+        trp.push_back((int32_t)de.size());
+        if (r >= nrows) continue;
+        const int64_t end = T.drow_ptr[q0 + r + 1];
+        while (cur[r] < end && T.d_slot[cur[r]] < s_hi) {
+          const int64_t e = cur[r];
+          int2 v;
+          v.x = T.d_slot[e] - (int32_t)(t * TW);
+          v.y = *reinterpret_cast<const int32_t*>(&A.val[T.d_cidx[e]]);
+          de.push_back(v);
+          deo.push_back(d_out[e]);
+          ++cur[r];
+        }
+      }
+      trp.push_back((int32_t)de.size());
+    }
+    ntiles_total += nt;
+    const int64_t nunits = (nt + kMaxUnitTiles - 1) / kMaxUnitTiles;
+    for (int64_t c = 0; c < nunits; ++c) {
+      const int64_t t0 = c * kMaxUnitTiles, t1 = std::min(nt, t0 + kMaxUnitTiles);
+      DUnit u;
+      u.q0 = (int32_t)q0;
+      u.nrows = (int32_t)nrows;
+      u.tile0 = (int32_t)(tile_base + t0);
+      u.ntiles = (int32_t)(t1 - t0);
+      u.dc0 = (int32_t)(dc0 + t0 * TW);
+      u.ncols = (int32_t)(std::min(nd, t1 * TW) - t0 * TW);
+      u.split = nunits > 1 ? (int32_t)(n_dslots + c) : -1;
+      u.pad = 0;
+      units.push_back(u);
+      if (nunits > 1) dsplit.push_back(make_int2((int)n_dslots, (int)nunits));
+    }
+    if (nunits > 1) n_dslots += nunits;
   }
-  P.n_dpanels = (int64_t)dp.size();
+  P.n_units = (int64_t)units.size();
   P.max_dense_per_panel = maxd;
-  P.tile_cols = h->params.tile_cols;
+  P.tile_cols = TW;
   P.panel_rows = PR;
-  SR_TRY(P.dpanels.upload(dp, s));
+  P.n_dslots = n_dslots;
+  P.dscratch.release();
+  P.dscratch_k = 0;
+  SR_TRY(P.units.upload(units, s));
   SR_TRY(P.dense_cols.upload(T.dense_cols, s));
+  SR_TRY(P.trp.upload(trp, s));
+  SR_TRY(P.d_ent.upload(de, s));
+  SR_TRY(P.d_oidx.upload(deo, s));
+  if (n_dslots > 0) {
+    SR_TRY(P.dsplit_info.upload(dsplit, s));
+    SR_TRY(P.dsplit_counter.alloc((size_t)n_dslots));
+    SR_CUDA_TRY(cudaMemsetAsync(P.dsplit_counter.p, 0, n_dslots * sizeof(int32_t), s));
+  }
   {
     std::vector<int32_t> drp((size_t)M + 1);
     for (int64_t q = 0; q <= M; ++q) drp[q] = (int32_t)T.drow_ptr[q];
     SR_TRY(P.drow_ptr.upload(drp, s));
-    std::vector<int2> de((size_t)T.n_dense());
-#pragma omp parallel for schedule(static)
-    for (int64_t e = 0; e < T.n_dense(); ++e) {
-      de[e].x = T.d_slot[e];
-      de[e].y = *reinterpret_cast<const int32_t*>(&A.val[T.d_cidx[e]]);
-    }
-    SR_TRY(P.d_ent.upload(de, s));
-    SR_TRY(P.d_oidx.upload(d_out, s));
     std::vector<int32_t> pout((size_t)M);
     for (int64_t q = 0; q < M; ++q) pout[q] = sharded ? (int32_t)(q - q0s) : perm1[q];
     SR_TRY(P.pos_xrow.upload(perm1, s));
@@ -256,15 +306,15 @@ int build_exec_plan(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s) {
   sparse_traffic(ib, n_nonzero, (int64_t)ib.items.size() - n_nonzero, se, A.N, tm);
   {
     std::vector<uint8_t> seen((size_t)A.N, 0);
-    for (const DPanel& d : dp) {
-      tm.dense_col_loads += d.dc1 - d.dc0;
-      for (int32_t k = d.dc0; k < d.dc1; ++k)
+    for (const DUnit& d : units) {
+      tm.dense_col_loads += d.ncols;
+      for (int32_t k = d.dc0; k < d.dc0 + d.ncols; ++k)
         if (!seen[T.dense_cols[k]]) {
           seen[T.dense_cols[k]] = 1;
           ++tm.dense_distinct_cols;
         }
     }
-    tm.dense_panels = (int64_t)dp.size();
+    tm.dense_panels = (int64_t)units.size();
     for (int64_t q = q0s; q < q1s; ++q) {
       const bool d = T.drow_ptr[q + 1] > T.drow_ptr[q], r = T.rrow_ptr[q + 1] > T.rrow_ptr[q];
       tm.dense_nnz += T.drow_ptr[q + 1] - T.drow_ptr[q];

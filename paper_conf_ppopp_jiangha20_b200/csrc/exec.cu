@@ -93,7 +93,7 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 
 // ------------------------------------------------------------------ phase S: SpMM
 template <int LPG, int VEC, int U>
-__global__ void __launch_bounds__(256) spmm_sparse_kernel(
+__global__ void __launch_bounds__(256, 4) spmm_sparse_kernel(
     const Item* __restrict__ items, const uint32_t* __restrict__ meta, int64_t n_items,
     const int2* __restrict__ ent, const float* __restrict__ B, int64_t ldb, float* __restrict__ C,
     int64_t ldc, int K, float* __restrict__ scratch, const int2* __restrict__ split_info,
@@ -236,232 +236,266 @@ __global__ void __launch_bounds__(256) sddmm_sparse_kernel(
 }
 
 // ------------------------------------------------------------------ phase D
-constexpr int kDenseWarps = 8;  // phase-D CTA = 8 warps; RPW = panel rows per warp (8 or 16)
+// Work unit = up to kMaxUnitTiles consecutive tiles of one panel (DUnit).  Entries are
+// stored tile-major: tile t, panel row r -> ent[trp[t·(P+1)+r] .. trp[t·(P+1)+r+1]) with
+// the slot relative to the tile.  A dedicated producer warp streams the unit's tiles
+// through an NST-stage shared-memory ring with cp.async.bulk (one 16-byte-aligned copy of
+// KC columns per dense column) and full/empty mbarriers, so consumer warps never meet at
+// a CTA barrier.  Consumer warp w owns the contiguous panel rows [w·RPW, (w+1)·RPW): its
+// entries of one tile are contiguous, so one coalesced load brings them in.
+constexpr int kDenseWarps = 8;  // consumer warps per phase-D CTA (+1 producer warp)
+constexpr int kStages = 3;
 
-// SpMM dense tiles.  Dynamic smem: 2 stages × SW slots × KC floats.
-template <int LPG, int VEC, int U, int kRPW, bool kBulk>
-__global__ void __launch_bounds__(256, 1) spmm_dense_kernel(
-    const DPanel* __restrict__ panels, const int32_t* __restrict__ dense_cols,
-    const int32_t* __restrict__ drow_ptr, const int2* __restrict__ d_ent,
-    const int32_t* __restrict__ pos_out, const float* __restrict__ B, int64_t ldb,
-    float* __restrict__ C, int64_t ldc, int K, int SW) {
-  constexpr int G = 32 / LPG;
-  constexpr int KC = LPG * VEC;
-  extern __shared__ __align__(128) float smem[];
-  __shared__ uint64_t full[2];
-  const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
-  const int warp = threadIdx.x >> 5, W = blockDim.x >> 5;
-  const DPanel pn = panels[blockIdx.x];
-  const int nd = pn.dc1 - pn.dc0;
-  const int ntile = (nd + SW - 1) / SW;
-  if (kBulk && threadIdx.x == 0) {
-    mbar_init(&full[0], 1);
-    mbar_init(&full[1], 1);
-    fence_mbar_init();
-  }
-  __syncthreads();
-  int tcount = 0;  // tiles issued so far (stage = tcount & 1, parity = (tcount >> 1) & 1)
-  for (int k0 = 0; k0 < K; k0 += KC) {
-    const int kw = min(KC, K - k0);  // columns staged per slot
-    auto issue = [&](int t, int st) {
-      const int s0 = t * SW, ns = min(SW, nd - s0);
-      float* dst = smem + (size_t)st * SW * KC;
-      if (kBulk) {
-        if (warp == 0) {
-          if (lane == 0) mbar_expect_tx(&full[st], (uint32_t)(ns * kw * 4));
-          __syncwarp();
-          for (int j = lane; j < ns; j += 32)
-            bulk_g2s(dst + (size_t)j * KC, B + (int64_t)dense_cols[pn.dc0 + s0 + j] * ldb + k0,
-                     (uint32_t)(kw * 4), &full[st]);
-        }
-      } else {
-        for (int idx = threadIdx.x; idx < ns * kw; idx += blockDim.x) {
-          const int j = idx / kw, k = idx % kw;
-          dst[(size_t)j * KC + k] = __ldg(B + (int64_t)dense_cols[pn.dc0 + s0 + j] * ldb + k0 + k);
-        }
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+// Producer warp: issue stage `st` with tile tt of pass k0.
+__device__ __forceinline__ void produce_tile(float* dst, const int32_t* __restrict__ cols, int ns, int KC,
+                                             int kw, const float* __restrict__ src, int64_t ld, int k0,
+                                             uint64_t* bar, int lane) {
+  if (lane == 0) mbar_expect_tx(bar, (uint32_t)(ns * kw * 4));
+  __syncwarp();
+  for (int j = lane; j < ns; j += 32)
+    bulk_g2s(dst + (size_t)j * KC, src + (int64_t)cols[j] * ld + k0, (uint32_t)(kw * 4), bar);
+}
+
+// Consumer-side iteration over the unit's (pass, tile) sequence.  Calls body(tile_smem,
+// tile_index, k0, kw) for every tile, and pass_end(k0) after the last tile of a pass.
+template <int VEC, bool kBulk, typename Body, typename PassEnd>
+__device__ __forceinline__ void dense_pipeline(const DUnit& u, const int32_t* __restrict__ dense_cols,
+                                               const float* __restrict__ src, int64_t ld, int K, int KC,
+                                               int TW, float* smem, uint64_t* full, uint64_t* empty,
+                                               Body body, PassEnd pass_end) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int npass = (K + KC - 1) / KC;
+  const int total = npass * u.ntiles;
+  if constexpr (kBulk) {
+    if (warp == kDenseWarps) {  // producer
+      for (int idx = 0; idx < total; ++idx) {
+        const int st = idx % kStages;
+        if (idx >= kStages) mbar_wait(&empty[st], ((idx - kStages) / kStages) & 1);
+        const int pass = idx / u.ntiles, tt = idx % u.ntiles;
+        const int k0 = pass * KC, kw = min(KC, K - k0), s0 = tt * TW;
+        produce_tile(smem + (size_t)st * TW * KC, dense_cols + u.dc0 + s0, min(TW, u.ncols - s0), KC, kw,
+                     src, ld, k0, &full[st], lane);
       }
-    };
-    int cur[kRPW], end[kRPW];
-    bool has[kRPW];
-    Frag<VEC> acc[kRPW];
-#pragma unroll
-    for (int i = 0; i < kRPW; ++i) {
-      const int r = warp + i * W;
-      if (r < pn.nrows) {
-        cur[i] = drow_ptr[pn.q0 + r];
-        end[i] = drow_ptr[pn.q0 + r + 1];
-      } else {
-        cur[i] = end[i] = 0;
-      }
-      has[i] = end[i] > cur[i];
-      acc[i].zero();
+      return;
     }
-    const int kk = k0 + lg * VEC;
-    const bool kv = kk < K;
-    if (ntile > 0) issue(0, tcount & 1);
-    for (int t = 0; t < ntile; ++t) {
-      const int st = (tcount + t) & 1;
-      if (t + 1 < ntile) issue(t + 1, (tcount + t + 1) & 1);
-      if (kBulk) mbar_wait(&full[st], ((tcount + t) >> 1) & 1);
-      else __syncthreads();
-      const float* tile = smem + (size_t)st * SW * KC;
-      const int s_lo = t * SW, s_hi = s_lo + SW;
-#pragma unroll
-      for (int i = 0; i < kRPW; ++i) {
-        while (cur[i] < end[i]) {
-          const int navail = min(32, end[i] - cur[i]);
-          const int2 my = lane < navail ? d_ent[cur[i] + lane] : make_int2(0x7fffffff, 0);
-          const unsigned inside = __ballot_sync(FULL, lane < navail && my.x < s_hi);
-          const int n = __popc(inside);
-          for (int base = 0; base < n; base += G * U) {
-            Frag<VEC> b[U];
-            float a[U];
-#pragma unroll
-            for (int u = 0; u < U; ++u) {
-              const int j = base + u * G + g;
-              const int slot = __shfl_sync(FULL, my.x, j & 31);
-              const float v = __int_as_float(__shfl_sync(FULL, my.y, j & 31));
-              const bool ok = j < n && kv;
-              a[u] = ok ? v : 0.f;
-              if (ok) b[u].load_s(tile + (size_t)(slot - s_lo) * KC + lg * VEC); else b[u].zero();
-            }
-#pragma unroll
-            for (int u = 0; u < U; ++u) acc[i].fma(a[u], b[u]);
-          }
-          cur[i] += n;
-          if (n < navail) break;
-        }
-      }
-      __syncthreads();  // stage st may be overwritten by the next issue
+    for (int idx = 0; idx < total; ++idx) {
+      const int st = idx % kStages;
+      mbar_wait(&full[st], (idx / kStages) & 1);
+      const int pass = idx / u.ntiles, tt = idx % u.ntiles;
+      const int k0 = pass * KC;
+      body(smem + (size_t)st * TW * KC, u.tile0 + tt, k0, min(KC, K - k0));
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[st]);
+      if (tt == u.ntiles - 1) pass_end(k0);
     }
-    tcount += ntile;
-#pragma unroll
-    for (int i = 0; i < kRPW; ++i) {
-#pragma unroll
-      for (int off = LPG; off < 32; off <<= 1) acc[i].xor_add(off);
-      const int r = warp + i * W;
-      if (has[i] && g == 0 && kv) acc[i].store_cs(C + (int64_t)pos_out[pn.q0 + r] * ldc + kk);
+  } else {
+    for (int idx = 0; idx < total; ++idx) {
+      const int pass = idx / u.ntiles, tt = idx % u.ntiles;
+      const int k0 = pass * KC, kw = min(KC, K - k0), s0 = tt * TW, ns = min(TW, u.ncols - s0);
+      __syncthreads();
+      for (int i = threadIdx.x; i < ns * kw; i += blockDim.x) {
+        const int j = i / kw, k = i % kw;
+        smem[(size_t)j * KC + k] = __ldg(src + (int64_t)dense_cols[u.dc0 + s0 + j] * ld + k0 + k);
+      }
+      __syncthreads();
+      if (warp < kDenseWarps) {
+        body(smem, u.tile0 + tt, k0, kw);
+        if (tt == u.ntiles - 1) pass_end(k0);
+      }
     }
   }
 }
 
-// SDDMM dense tiles.  Slots hold the full (padded) K of each Y row: NCH × KC floats.
-template <int LPG, int VEC, int U, int NCH, int kRPW, bool kBulk>
-__global__ void __launch_bounds__(256, 1) sddmm_dense_kernel(
-    const DPanel* __restrict__ panels, const int32_t* __restrict__ dense_cols,
-    const int32_t* __restrict__ drow_ptr, const int2* __restrict__ d_ent,
-    const int32_t* __restrict__ d_oidx, const int32_t* __restrict__ pos_xrow,
-    const float* __restrict__ X, int64_t ldx, const float* __restrict__ Y, int64_t ldy, int K,
-    int SW, float* __restrict__ out) {
-  constexpr int G = 32 / LPG;
-  constexpr int KC = LPG * VEC;
-  constexpr int SLOT = NCH * KC;
-  extern __shared__ __align__(128) float smem[];
-  __shared__ uint64_t full[2];
-  const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
-  const int warp = threadIdx.x >> 5, W = blockDim.x >> 5;
-  const DPanel pn = panels[blockIdx.x];
-  const int nd = pn.dc1 - pn.dc0;
-  const int ntile = (nd + SW - 1) / SW;
-  if (kBulk && threadIdx.x == 0) {
-    mbar_init(&full[0], 1);
-    mbar_init(&full[1], 1);
+__device__ __forceinline__ void dense_init_barriers(uint64_t* full, uint64_t* empty) {
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < kStages; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], kDenseWarps);
+    }
     fence_mbar_init();
   }
   __syncthreads();
-  auto issue = [&](int t, int st) {
-    const int s0 = t * SW, ns = min(SW, nd - s0);
-    float* dst = smem + (size_t)st * SW * SLOT;
-    if (kBulk) {
-      if (warp == 0) {
-        if (lane == 0) mbar_expect_tx(&full[st], (uint32_t)(ns * K * 4));
-        __syncwarp();
-        for (int j = lane; j < ns; j += 32)
-          bulk_g2s(dst + (size_t)j * SLOT, Y + (int64_t)dense_cols[pn.dc0 + s0 + j] * ldy,
-                   (uint32_t)(K * 4), &full[st]);
-      }
-    } else {
-      for (int idx = threadIdx.x; idx < ns * K; idx += blockDim.x) {
-        const int j = idx / K, k = idx % K;
-        dst[(size_t)j * SLOT + k] = __ldg(Y + (int64_t)dense_cols[pn.dc0 + s0 + j] * ldy + k);
+}
+
+// SpMM dense tiles.
+template <int LPG, int VEC, int U, int RPW, bool kBulk>
+__global__ void __launch_bounds__((kDenseWarps + 1) * 32, 2) spmm_dense_kernel(
+    const DUnit* __restrict__ units, const int32_t* __restrict__ dense_cols, const int32_t* __restrict__ trp,
+    const int2* __restrict__ ent, const int32_t* __restrict__ drow_ptr, const int32_t* __restrict__ pos_out,
+    const float* __restrict__ B, int64_t ldb, float* __restrict__ C, int64_t ldc, int K, int TW, int P,
+    float* __restrict__ scratch, const int2* __restrict__ split_info, int* __restrict__ split_counter) {
+  constexpr int G = 32 / LPG;
+  constexpr int KC = LPG * VEC;
+  extern __shared__ __align__(128) float smem[];
+  __shared__ uint64_t full[kStages], empty[kStages];
+  const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
+  const int warp = threadIdx.x >> 5;
+  const DUnit u = units[blockIdx.x];
+  dense_init_barriers(full, empty);
+  const int r0 = warp * RPW;
+  Frag<VEC> acc[RPW];
+#pragma unroll
+  for (int i = 0; i < RPW; ++i) acc[i].zero();
+  auto body = [&](const float* tile, int t, int k0, int kw) {
+    if (r0 >= u.nrows) return;
+    const int kk = k0 + lg * VEC;
+    const bool kv = lg * VEC < kw;
+    const int32_t* rp = trp + (int64_t)t * (P + 1) + r0;
+    const int bnd = lane <= RPW ? __ldg(rp + lane) : 0;  // row bounds of this warp's rows
+    const int e_lo = __shfl_sync(FULL, bnd, 0), e_hi = __shfl_sync(FULL, bnd, RPW);
+    (void)kk;
+    for (int e = e_lo; e < e_hi; e += 32) {
+      const int n = min(32, e_hi - e);
+      const int2 my = lane < n ? __ldcs(ent + e + lane) : make_int2(0, 0);
+#pragma unroll
+      for (int i = 0; i < RPW; ++i) {
+        // entries of row r0+i inside this 32-entry chunk: [a, b) in lane space
+        const int a = max(0, __shfl_sync(FULL, bnd, i) - e), b = min(n, __shfl_sync(FULL, bnd, i + 1) - e);
+        for (int base = a; base < b; base += G * U) {
+          Frag<VEC> bv[U];
+          float av[U];
+#pragma unroll
+          for (int uu = 0; uu < U; ++uu) {
+            const int j = base + uu * G + g;
+            const int slot = __shfl_sync(FULL, my.x, j & 31);
+            const float v = __int_as_float(__shfl_sync(FULL, my.y, j & 31));
+            const bool ok = j < b && kv;
+            av[uu] = ok ? v : 0.f;
+            if (ok) bv[uu].load_s(tile + (size_t)slot * KC + lg * VEC); else bv[uu].zero();
+          }
+#pragma unroll
+          for (int uu = 0; uu < U; ++uu) acc[i].fma(av[uu], bv[uu]);
+        }
       }
     }
   };
-  int cur[kRPW], end[kRPW];
+  auto pass_end = [&](int k0) {
+    const int kk = k0 + lg * VEC;
+    const bool kv = kk < K;
 #pragma unroll
-  for (int i = 0; i < kRPW; ++i) {
-    const int r = warp + i * W;
-    if (r < pn.nrows) {
-      cur[i] = drow_ptr[pn.q0 + r];
-      end[i] = drow_ptr[pn.q0 + r + 1];
-    } else {
-      cur[i] = end[i] = 0;
-    }
-  }
-  if (ntile > 0) issue(0, 0);
-  for (int t = 0; t < ntile; ++t) {
-    const int st = t & 1;
-    if (t + 1 < ntile) issue(t + 1, (t + 1) & 1);
-    if (kBulk) mbar_wait(&full[st], (t >> 1) & 1);
-    else __syncthreads();
-    const float* tile = smem + (size_t)st * SW * SLOT;
-    const int s_lo = t * SW, s_hi = s_lo + SW;
+    for (int i = 0; i < RPW; ++i) {
 #pragma unroll
-    for (int i = 0; i < kRPW; ++i) {
-      if (cur[i] >= end[i]) continue;
-      const int r = warp + i * W;
-      const int xr = pos_xrow[pn.q0 + r];
-      Frag<VEC> x[NCH];
-#pragma unroll
-      for (int c = 0; c < NCH; ++c) {
-        const int kk = c * KC + lg * VEC;
-        if (kk < K) x[c].load_g(X + (int64_t)xr * ldx + kk); else x[c].zero();
+      for (int off = LPG; off < 32; off <<= 1) acc[i].xor_add(off);
+      const int r = r0 + i;
+      if (r < u.nrows && g == 0 && kv) {
+        if (u.split >= 0)
+          acc[i].store(scratch + ((int64_t)u.split * P + r) * K + kk);
+        else if (drow_ptr[u.q0 + r + 1] > drow_ptr[u.q0 + r])
+          acc[i].store_cs(C + (int64_t)pos_out[u.q0 + r] * ldc + kk);
       }
-      while (cur[i] < end[i]) {
-        const int navail = min(32, end[i] - cur[i]);
-        const int2 my = lane < navail ? d_ent[cur[i] + lane] : make_int2(0x7fffffff, 0);
-        const int myo = lane < navail ? d_oidx[cur[i] + lane] : 0;
-        const unsigned inside = __ballot_sync(FULL, lane < navail && my.x < s_hi);
-        const int n = __popc(inside);
-        for (int base = 0; base < n; base += G * U) {
+      acc[i].zero();
+    }
+  };
+  dense_pipeline<VEC, kBulk>(u, dense_cols, B, ldb, K, KC, TW, smem, full, empty, body, pass_end);
+  if (u.split >= 0) {
+    // giant panel split over several units: the last unit to finish sums the chunk
+    // partials in chunk order (deterministic) and writes the panel's dense rows
+    __shared__ int last;
+    __threadfence();
+    __syncthreads();
+    const int2 si = split_info[u.split];
+    if (threadIdx.x == 0) last = (atomicAdd(split_counter + si.x, 1) == si.y - 1);
+    __syncthreads();
+    if (!last) return;
+    __threadfence();
+    for (int r = warp; r < u.nrows; r += kDenseWarps + 1) {
+      if (drow_ptr[u.q0 + r + 1] == drow_ptr[u.q0 + r]) continue;
+      for (int k = lane * VEC; k < K; k += 32 * VEC) {
+        Frag<VEC> s;
+        s.zero();
+        for (int c = 0; c < si.y; ++c) {
+          Frag<VEC> part;
+          part.load_cg(scratch + ((int64_t)(si.x + c) * P + r) * K + k);
+          s.add(part);
+        }
+        s.store_cs(C + (int64_t)pos_out[u.q0 + r] * ldc + k);
+      }
+    }
+    if (threadIdx.x == 0) split_counter[si.x] = 0;
+  }
+}
+
+// SDDMM dense tiles: per K pass, X fragments of the warp's rows stay in registers and every
+// tile nnz gets one dot product from shared memory; passes after the first accumulate into
+// out (same lane, same order: deterministic).
+template <int LPG, int VEC, int U, int RPW, bool kBulk>
+__global__ void __launch_bounds__((kDenseWarps + 1) * 32, 2) sddmm_dense_kernel(
+    const DUnit* __restrict__ units, const int32_t* __restrict__ dense_cols, const int32_t* __restrict__ trp,
+    const int2* __restrict__ ent, const int32_t* __restrict__ d_oidx, const int32_t* __restrict__ pos_xrow,
+    const float* __restrict__ X, int64_t ldx, const float* __restrict__ Y, int64_t ldy, int K, int TW, int P,
+    float* __restrict__ out) {
+  constexpr int G = 32 / LPG;
+  constexpr int KC = LPG * VEC;
+  extern __shared__ __align__(128) float smem[];
+  __shared__ uint64_t full[kStages], empty[kStages];
+  const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
+  const int warp = threadIdx.x >> 5;
+  const DUnit u = units[blockIdx.x];
+  dense_init_barriers(full, empty);
+  const int r0 = warp * RPW;
+  Frag<VEC> x[RPW];
+  int xk0 = -1;
+  auto body = [&](const float* tile, int t, int k0, int kw) {
+    if (r0 >= u.nrows) return;
+    const bool kv = lg * VEC < kw;
+    if (k0 != xk0) {  // new K pass: this warp's X fragments
+#pragma unroll
+      for (int i = 0; i < RPW; ++i) {
+        if (r0 + i < u.nrows && kv) x[i].load_g(X + (int64_t)pos_xrow[u.q0 + r0 + i] * ldx + k0 + lg * VEC);
+        else x[i].zero();
+      }
+      xk0 = k0;
+    }
+    const int32_t* rp = trp + (int64_t)t * (P + 1) + r0;
+    const int bnd = lane <= RPW ? __ldg(rp + lane) : 0;
+    const int e_lo = __shfl_sync(FULL, bnd, 0), e_hi = __shfl_sync(FULL, bnd, RPW);
+    for (int e = e_lo; e < e_hi; e += 32) {
+      const int n = min(32, e_hi - e);
+      const int2 my = lane < n ? __ldcs(ent + e + lane) : make_int2(0, 0);
+      const int myo = lane < n ? __ldcs(d_oidx + e + lane) : 0;
+#pragma unroll
+      for (int i = 0; i < RPW; ++i) {
+        const int a = max(0, __shfl_sync(FULL, bnd, i) - e), b = min(n, __shfl_sync(FULL, bnd, i + 1) - e);
+        for (int base = a; base < b; base += G * U) {
           float part[U];
 #pragma unroll
-          for (int u = 0; u < U; ++u) {
-            const int j = base + u * G + g;
+          for (int uu = 0; uu < U; ++uu) {
+            const int j = base + uu * G + g;
             const int slot = __shfl_sync(FULL, my.x, j & 31);
             float d = 0.f;
-            if (j < n) {
-#pragma unroll
-              for (int c = 0; c < NCH; ++c) {
-                const int kk = c * KC + lg * VEC;
-                if (kk < K) {
-                  Frag<VEC> y;
-                  y.load_s(tile + (size_t)(slot - s_lo) * SLOT + kk);
-                  d += x[c].dot(y);
-                }
-              }
+            if (j < b && kv) {
+              Frag<VEC> y;
+              y.load_s(tile + (size_t)slot * KC + lg * VEC);
+              d = x[i].dot(y);
             }
-            part[u] = d;
+            part[uu] = d;
           }
 #pragma unroll
-          for (int u = 0; u < U; ++u) {
+          for (int uu = 0; uu < U; ++uu) {
 #pragma unroll
-            for (int off = LPG / 2; off > 0; off >>= 1) part[u] += __shfl_xor_sync(FULL, part[u], off);
+            for (int off = LPG / 2; off > 0; off >>= 1) part[uu] += __shfl_xor_sync(FULL, part[uu], off);
           }
 #pragma unroll
-          for (int u = 0; u < U; ++u) {
-            const int j = base + u * G + g;
+          for (int uu = 0; uu < U; ++uu) {
+            const int j = base + uu * G + g;
             const float v = __int_as_float(__shfl_sync(FULL, my.y, j & 31));
             const int o = __shfl_sync(FULL, myo, j & 31);
-            if (lg == 0 && j < n) __stcs(out + o, v * part[u]);
+            if (lg == 0 && j < b) {
+              float res = v * part[uu];
+              if (k0 > 0) res += out[o];
+              out[o] = res;
+            }
           }
         }
-        cur[i] += n;
-        if (n < navail) break;
       }
     }
-    __syncthreads();
-  }
+  };
+  auto pass_end = [&](int) {};
+  dense_pipeline<VEC, kBulk>(u, dense_cols, Y, ldy, K, KC, TW, smem, full, empty, body, pass_end);
 }
 
 // ------------------------------------------------------------------ host dispatch
@@ -471,7 +505,6 @@ inline int next_pow2(int x) {
   return p;
 }
 
-constexpr int kStageBytes = 48 * 1024;
 constexpr int kSparseWarps = 8;
 
 template <int LPG, int VEC>
@@ -481,13 +514,18 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
   constexpr int KC = LPG * VEC;
   constexpr int U = (LPG == 32) ? 8 : 4;  // gathers in flight per lane (phase S)
   constexpr int UD = 4;                   // shared-memory reads in flight per lane (phase D)
-  if (P.n_dpanels > 0) {
-    const int SW = std::max(1, std::min(P.tile_cols, kStageBytes / (KC * 4)));
-    const size_t smem = (size_t)2 * SW * KC * sizeof(float);
+  if (P.n_units > 0) {
+    const int TW = P.tile_cols;
+    const size_t smem = (size_t)kStages * TW * KC * sizeof(float);
+    if (P.n_dslots > 0 && P.dscratch_k < K) {
+      SR_TRY(P.dscratch.alloc((size_t)P.n_dslots * P.panel_rows * K));
+      P.dscratch_k = K;
+    }
     auto launch = [&](auto kern) -> int {
       SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-      kern<<<(unsigned)P.n_dpanels, kDenseWarps * 32, smem, s>>>(P.dpanels.p, P.dense_cols.p, P.drow_ptr.p,
-                                                                P.d_ent.p, P.pos_out.p, B, ldb, C, ldc, (int)K, SW);
+      kern<<<(unsigned)P.n_units, (kDenseWarps + 1) * 32, smem, s>>>(
+          P.units.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.drow_ptr.p, P.pos_out.p, B, ldb, C, ldc, (int)K, TW,
+          P.panel_rows, P.dscratch.p, P.dsplit_info.p, P.dsplit_counter.p);
       SR_CUDA_TRY(cudaGetLastError());
       return SR_OK;
     };
@@ -524,24 +562,24 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
   DevPlan& P = h->plan;
   constexpr int KC = LPG * VEC;
   constexpr int U = (LPG == 32) ? 4 : 2;
-  if (P.n_dpanels > 0) {
-    const int slot_floats = NCH * KC;
-    const int SW = std::max(1, std::min(P.tile_cols, kStageBytes / (slot_floats * 4)));
-    const size_t smem = (size_t)2 * SW * slot_floats * sizeof(float);
+  if (P.n_units > 0) {
+    const int TW = P.tile_cols;
+    const size_t smem = (size_t)kStages * TW * KC * sizeof(float);
     auto launch = [&](auto kern) -> int {
       SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-      kern<<<(unsigned)P.n_dpanels, kDenseWarps * 32, smem, s>>>(P.dpanels.p, P.dense_cols.p, P.drow_ptr.p,
-                                                                P.d_ent.p, P.d_oidx.p, P.pos_xrow.p, X, ldx, Y,
-                                                                ldy, (int)K, SW, out);
+      kern<<<(unsigned)P.n_units, (kDenseWarps + 1) * 32, smem, s>>>(
+          P.units.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.d_oidx.p, P.pos_xrow.p, X, ldx, Y, ldy, (int)K, TW,
+          P.panel_rows, out);
       SR_CUDA_TRY(cudaGetLastError());
       return SR_OK;
     };
+    constexpr int UD = 4;
     if (P.profiling) SR_TRY(prof_begin(P, 3, s));
     if (VEC == 4) {
-      if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, U, NCH, 8, true>));
-      else SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, U, NCH, 16, true>));
+      if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, 8, true>));
+      else SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, 16, true>));
     } else {
-      SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, U, NCH, 16, false>));
+      SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, 16, false>));
     }
     if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;

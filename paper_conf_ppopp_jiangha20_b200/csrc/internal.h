@@ -103,21 +103,32 @@ constexpr uint32_t kItemRMW = 1u << 31;    // C[out] += partial (row also has de
 constexpr uint32_t kItemSplit = 1u << 30;  // partial of a split long row -> scratch slot
 constexpr uint32_t kItemSlotMask = (1u << 30) - 1;
 
-// Phase-D work unit: one CTA per panel with at least one dense column.
-struct __align__(16) DPanel {
-  int32_t q0, nrows;  // positions [q0, q0+nrows)
-  int32_t dc0, dc1;   // dense_cols[dc0, dc1) = D_p
+// Phase-D work unit (one CTA): up to kMaxUnitTiles consecutive tiles of one panel.
+struct __align__(16) DUnit {
+  int32_t q0, nrows;      // panel positions [q0, q0+nrows)
+  int32_t tile0, ntiles;  // global tile ids [tile0, tile0+ntiles)
+  int32_t dc0, ncols;     // dense_cols[dc0, dc0+ncols): the columns staged by this unit
+  int32_t split;          // -1: the unit covers its whole panel; else its partial-sum slot
+  int32_t pad;
 };
+constexpr int kMaxUnitTiles = 16;
+constexpr int kMaxExecTile = 64;
 
 // Device-resident execution plan.
 struct DevPlan {
   // phase D
-  DevBuf<DPanel> dpanels;
-  int64_t n_dpanels = 0;
+  DevBuf<DUnit> units;
+  int64_t n_units = 0;
   DevBuf<int32_t> dense_cols;
-  DevBuf<int32_t> drow_ptr;   // positions -> offsets into d_ent
-  DevBuf<int2> d_ent;         // {slot, __float_as_int(val)}
-  DevBuf<int32_t> d_oidx;     // SDDMM output index per dense nnz
+  DevBuf<int32_t> trp;        // per tile: panel_rows+1 offsets into d_ent (tile-major layout)
+  DevBuf<int32_t> drow_ptr;   // positions -> dense nnz offsets (only "row has dense nnz" is used)
+  DevBuf<int2> d_ent;         // tile-major {slot in tile, __float_as_int(val)}
+  DevBuf<int32_t> d_oidx;     // SDDMM output index per dense nnz (tile-major)
+  DevBuf<int2> dsplit_info;   // per split unit: {first slot, nchunks}
+  DevBuf<int32_t> dsplit_counter;
+  int64_t n_dslots = 0;
+  DevBuf<float> dscratch;     // n_dslots × panel_rows × dscratch_k
+  int64_t dscratch_k = 0;
   DevBuf<int32_t> pos_xrow;   // position -> original row
   DevBuf<int32_t> pos_out;    // position -> SpMM output row
   // phase S
