@@ -163,6 +163,15 @@ int sr_shard_rows(sr_csr h, int32_t* rows_out, int64_t cap, int64_t* len);
 /* Original nnz ids of this handle's shard, in the packed order sr_sddmm writes. */
 int sr_shard_nnz_ids(sr_csr h, int64_t* ids_out, int64_t cap, int64_t* len);
 
+/* Gather helpers for sharded plans: after an all-gather of the packed shard
+ * outputs, scatter them back to original positions.  All pointers are DEVICE memory.
+ *   sr_scatter_rows  : dst[rows[r], 0:K] = src[r, 0:K] for r < n (rows[r] < 0 skipped)
+ *   sr_scatter_values: dst[ids[i]] = src[i] for i < n (ids[i] < 0 skipped)
+ * Asynchronous on `stream`.  Errors: SR_EINVAL, SR_ECUDA. */
+int sr_scatter_rows(const float* src, int64_t lds, const int32_t* rows, int64_t n, int64_t K, float* dst,
+                    int64_t ldd, sr_stream stream);
+int sr_scatter_values(const float* src, const int64_t* ids, int64_t n, float* dst, sr_stream stream);
+
 /* Kernel launches the last sr_spmm / sr_sddmm call issued on this handle. */
 int sr_last_launch_count(sr_csr h, int32_t* n);
 

@@ -63,7 +63,8 @@ KERNEL_KINDS = {1: "spmm_dense_tiles", 2: "spmm_sparse_rows", 3: "sddmm_dense_ti
 EXPORTED = ("sr_csr_create", "sr_default_params", "sr_reorder", "sr_spmm", "sr_sddmm", "sr_destroy",
             "sr_get_perm", "sr_get_plan_stats", "sr_export_tiles", "sr_shard_rows", "sr_shard_nnz_ids",
             "sr_last_launch_count", "sr_last_error", "sr_host_cluster", "sr_host_partition", "sr_version",
-            "sr_get_traffic_model", "sr_set_profiling", "sr_last_kernel_times")
+            "sr_get_traffic_model", "sr_set_profiling", "sr_last_kernel_times", "sr_scatter_rows",
+            "sr_scatter_values")
 
 _lib = None
 
@@ -97,6 +98,8 @@ def lib():
         "sr_get_traffic_model": (C.c_int, [P, C.POINTER(TrafficModel)]),
         "sr_set_profiling": (C.c_int, [P, C.c_int]),
         "sr_last_kernel_times": (C.c_int, [P, P, P, i32, C.POINTER(i32)]),
+        "sr_scatter_rows": (C.c_int, [P, i64, P, i64, i64, P, i64, P]),
+        "sr_scatter_values": (C.c_int, [P, P, i64, P, P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -305,6 +308,19 @@ def host_partition(weights, G: int) -> np.ndarray:
     cuts = np.empty(G + 1, np.int64)
     _check(lib().sr_host_partition(w.size, pw, G, cuts.ctypes.data_as(C.c_void_p)))
     return cuts
+
+
+def scatter_rows(src, rows, dst, stream=None):
+    """dst[rows[r]] = src[r] on the device (rows: int32 CUDA tensor; -1 entries skipped)."""
+    _check(lib().sr_scatter_rows(_ptr(src), src.stride(0), _ptr(rows), rows.numel(), src.shape[1], _ptr(dst),
+                                 dst.stride(0), _stream(stream)))
+    return dst
+
+
+def scatter_values(src, ids, dst, stream=None):
+    """dst[ids[i]] = src[i] on the device (ids: int64 CUDA tensor; -1 entries skipped)."""
+    _check(lib().sr_scatter_values(_ptr(src), _ptr(ids), ids.numel(), _ptr(dst), _stream(stream)))
+    return dst
 
 
 def version() -> str:

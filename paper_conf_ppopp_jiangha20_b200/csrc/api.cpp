@@ -717,6 +717,18 @@ int sr_host_cluster(int64_t M, const int64_t* rowptr, const int32_t* colidx, int
   return SR_OK;
 }
 
+int sr_scatter_rows(const float* src, int64_t lds, const int32_t* rows, int64_t n, int64_t K, float* dst,
+                    int64_t ldd, sr_stream stream) {
+  if (n < 0 || K < 1 || lds < K || ldd < K || (n > 0 && (!src || !rows || !dst)))
+    return einval("sr_scatter_rows: bad argument");
+  return launch_scatter_rows(src, lds, rows, n, K, dst, ldd, (cudaStream_t)stream);
+}
+
+int sr_scatter_values(const float* src, const int64_t* ids, int64_t n, float* dst, sr_stream stream) {
+  if (n < 0 || (n > 0 && (!src || !ids || !dst))) return einval("sr_scatter_values: bad argument");
+  return launch_scatter_values(src, ids, n, dst, (cudaStream_t)stream);
+}
+
 int sr_host_partition(int64_t npanels, const int64_t* weights, int32_t G, int64_t* cuts) {
   if (npanels < 0 || G < 1 || !cuts || (npanels > 0 && !weights)) return einval("sr_host_partition: bad argument");
   partition_panels(npanels, weights, G, cuts);

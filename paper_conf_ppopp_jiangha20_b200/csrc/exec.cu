@@ -661,3 +661,36 @@ int launch_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64
 }
 
 }  // namespace sr
+
+// ------------------------------------------------------------------ gather helpers (a11)
+namespace sr {
+namespace {
+__global__ void scatter_rows_kernel(const float* __restrict__ src, int64_t lds, const int32_t* __restrict__ rows,
+                                    int64_t n, int64_t K, float* __restrict__ dst, int64_t ldd) {
+  const int64_t r = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  if (r >= n) return;
+  const int32_t d = rows[r];
+  if (d < 0) return;
+  for (int64_t k = threadIdx.x & 31; k < K; k += 32) dst[(int64_t)d * ldd + k] = src[r * lds + k];
+}
+__global__ void scatter_values_kernel(const float* __restrict__ src, const int64_t* __restrict__ ids, int64_t n,
+                                      float* __restrict__ dst) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n && ids[i] >= 0) dst[ids[i]] = src[i];
+}
+}  // namespace
+
+int launch_scatter_rows(const float* src, int64_t lds, const int32_t* rows, int64_t n, int64_t K, float* dst,
+                        int64_t ldd, cudaStream_t s) {
+  if (n == 0) return SR_OK;
+  scatter_rows_kernel<<<(unsigned)((n + 7) / 8), 256, 0, s>>>(src, lds, rows, n, K, dst, ldd);
+  SR_CUDA_TRY(cudaGetLastError());
+  return SR_OK;
+}
+int launch_scatter_values(const float* src, const int64_t* ids, int64_t n, float* dst, cudaStream_t s) {
+  if (n == 0) return SR_OK;
+  scatter_values_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(src, ids, n, dst);
+  SR_CUDA_TRY(cudaGetLastError());
+  return SR_OK;
+}
+}  // namespace sr

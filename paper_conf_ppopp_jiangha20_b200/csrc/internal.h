@@ -196,4 +196,7 @@ int launch_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, i
                 cudaStream_t s, int32_t* launches);
 int launch_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t ldy, int64_t K,
                  float* out, cudaStream_t s, int32_t* launches);
+int launch_scatter_rows(const float* src, int64_t lds, const int32_t* rows, int64_t n, int64_t K, float* dst,
+                        int64_t ldd, cudaStream_t s);
+int launch_scatter_values(const float* src, const int64_t* ids, int64_t n, float* dst, cudaStream_t s);
 }  // namespace sr

@@ -302,3 +302,50 @@ def test_rmat_full_size_sampled(env, oracle):
     ref_o, bound = oracle.sddmm(sub, X[rows], Y)
     err = np.abs(out[sel] - ref_o)
     assert not (err > TOL * bound + 1e-30).any()
+
+
+def test_scatter_helpers_reassemble_shards(env, oracle):
+    """The device scatter kernels (used by dist.gather_*) put packed shard outputs back."""
+    sr, torch = env
+    A = g.random_csr(400, 250, 0.03, 23, empty_frac=0.1)
+    K = 16
+    B = torch.from_numpy(g.dense(250, K)).cuda()
+    X = torch.from_numpy(g.dense(400, K, stream=1)).cuda()
+    Y = torch.from_numpy(g.dense(250, K, stream=2)).cuda()
+    C = torch.full((400, K), float("nan"), device="cuda")
+    out = torch.full((A.nnz,), float("nan"), device="cuda")
+    for r in range(2):
+        M = sr.SparseMatrix.from_csr(A)
+        M.reorder(sr.default_params(**_plan_kw(16, 1, 0), world=2, rank=r))
+        sr.scatter_rows(M.spmm(B), torch.from_numpy(M.shard_rows()).cuda(), C)
+        sr.scatter_values(M.sddmm(X, Y), torch.from_numpy(M.shard_nnz_ids()).cuda(), out)
+    torch.cuda.synchronize()
+    _spmm_check(oracle, A, B.cpu().numpy(), C.cpu().numpy())
+    _sddmm_check(oracle, A, X.cpu().numpy(), Y.cpu().numpy(), out.cpu().numpy())
+
+
+def test_dist_gather_single_rank_nccl(env, oracle):
+    """dist.gather_spmm / gather_sddmm through a real NCCL process group (world size 1)."""
+    sr, torch = env
+    import socket
+    import torch.distributed as tdist
+    from paper_conf_ppopp_jiangha20_b200 import dist
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    tdist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{port}", rank=0, world_size=1)
+    try:
+        A = g.random_csr(300, 200, 0.04, 5, empty_frac=0.1)
+        M = sr.SparseMatrix.from_csr(A)
+        M.reorder(sr.default_params(**_plan_kw(16, 1, 0)))
+        B = torch.from_numpy(g.dense(200, 32)).cuda()
+        X = torch.from_numpy(g.dense(300, 32, stream=1)).cuda()
+        Y = torch.from_numpy(g.dense(200, 32, stream=2)).cuda()
+        C = dist.gather_spmm(M, M.spmm(B))
+        out = dist.gather_sddmm(M, M.sddmm(X, Y))
+        torch.cuda.synchronize()
+        _spmm_check(oracle, A, B.cpu().numpy(), C.cpu().numpy())
+        _sddmm_check(oracle, A, X.cpu().numpy(), Y.cpu().numpy(), out.cpu().numpy())
+    finally:
+        tdist.destroy_process_group()
