@@ -189,19 +189,34 @@ int build_exec_plan(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s) {
       }
     }
   }
-  // phase D: tiles of tile_cols dense columns, tile-major entries, units of <= kMaxUnitTiles tiles
-  // execution tile width: the plan's tiles (tile_cols, reported in the metadata) are staged
-  // in sub-tiles of at most kMaxExecTile columns so two stages of K<=128 fit in 64 KB
+  if (!sharded) {  // single shard: outputs come back in the caller's order
+    std::iota(h->shard_rows.begin(), h->shard_rows.end(), 0);
+    std::iota(h->shard_nnz_ids.begin(), h->shard_nnz_ids.end(), 0);
+  }
+  // phase D: execution tiles of <= kMaxExecTile dense columns (the plan's tiles of tile_cols
+  // columns are reported in the metadata and staged in sub-tiles); each tile's entries are
+  // stored tile-major with panel-row offsets (trp) relative to the tile's entry block; a
+  // tile with more than kMaxTileEntries entries is split by rows into virtual tiles that
+  // stage the same columns; units of <= kMaxUnitTiles virtual tiles (giant panels -> split
+  // units with an ordered combine).
   const int32_t TW = std::min(h->params.tile_cols, kMaxExecTile);
+  const int32_t TS = (PR + 1 + 3) / 4 * 4;
   std::vector<DUnit> units;
+  std::vector<VTile> vtiles;
   std::vector<int2> dsplit;
   std::vector<int32_t> trp;
   std::vector<int2> de;
   std::vector<int32_t> deo;
-  de.reserve((size_t)T.n_dense());
-  deo.reserve((size_t)T.n_dense());
-  int64_t maxd = 0, ntiles_total = 0, n_dslots = 0;
-  std::vector<int64_t> cur((size_t)PR);
+  de.reserve((size_t)T.n_dense() + T.n_dense() / 4);
+  deo.reserve((size_t)T.n_dense() + T.n_dense() / 4);
+  int64_t maxd = 0, n_dslots = 0;
+  std::vector<int64_t> cur((size_t)PR), stop((size_t)PR);
+  auto pad4 = [&]() {
+    while (de.size() % 4) {
+      de.push_back(make_int2(0, 0));
+      deo.push_back(-1);
+    }
+  };
   for (int64_t p = pb; p < pe; ++p) {
     const int64_t dc0 = T.dense_ptr[p], dc1 = T.dense_ptr[p + 1];
     if (dc1 == dc0) continue;
@@ -209,51 +224,71 @@ int build_exec_plan(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s) {
     const int64_t nd = dc1 - dc0, nt = (nd + TW - 1) / TW;
     maxd = std::max(maxd, nd);
     for (int64_t r = 0; r < nrows; ++r) cur[r] = T.drow_ptr[q0 + r];
-    const int64_t tile_base = ntiles_total;
+    const int64_t vt_first = (int64_t)vtiles.size();
     for (int64_t t = 0; t < nt; ++t) {
       const int64_t s_hi = (t + 1) * TW;
-      for (int64_t r = 0; r < PR; ++r) {
-        trp.push_back((int32_t)de.size());
-        if (r >= nrows) continue;
+      for (int64_t r = 0; r < nrows; ++r) {
+        stop[r] = cur[r];
         const int64_t end = T.drow_ptr[q0 + r + 1];
-        while (cur[r] < end && T.d_slot[cur[r]] < s_hi) {
-          const int64_t e = cur[r];
-          int2 v;
-          v.x = T.d_slot[e] - (int32_t)(t * TW);
-          v.y = *reinterpret_cast<const int32_t*>(&A.val[T.d_cidx[e]]);
-          de.push_back(v);
-          deo.push_back(d_out[e]);
-          ++cur[r];
-        }
+        while (stop[r] < end && T.d_slot[stop[r]] < s_hi) ++stop[r];
       }
-      trp.push_back((int32_t)de.size());
+      int64_t ra = 0;
+      while (ra < std::max<int64_t>(nrows, 1)) {
+        int64_t rb = ra, cnt = 0;
+        while (rb < nrows && cnt + (stop[rb] - cur[rb]) <= kMaxTileEntries) cnt += stop[rb] - cur[rb], ++rb;
+        if (rb == ra) rb = ra + 1;  // cannot happen (a row has <= TW entries per tile)
+        pad4();
+        VTile v;
+        v.ent0 = (int32_t)de.size();
+        v.col0 = (int32_t)(dc0 + t * TW);
+        v.ncols = (int32_t)(std::min(nd, s_hi) - t * TW);
+        int32_t off = 0;
+        for (int64_t r = 0; r < TS; ++r) {
+          trp.push_back(off);
+          if (r >= ra && r < rb && r < nrows) {
+            for (int64_t e = cur[r]; e < stop[r]; ++e) {
+              int2 x;
+              x.x = T.d_slot[e] - (int32_t)(t * TW);
+              x.y = *reinterpret_cast<const int32_t*>(&A.val[T.d_cidx[e]]);
+              de.push_back(x);
+              deo.push_back(d_out[e]);
+              ++off;
+            }
+          }
+        }
+        pad4();
+        v.nent = (int32_t)de.size() - v.ent0;
+        vtiles.push_back(v);
+        ra = rb;
+      }
+      for (int64_t r = 0; r < nrows; ++r) cur[r] = stop[r];
     }
-    ntiles_total += nt;
-    const int64_t nunits = (nt + kMaxUnitTiles - 1) / kMaxUnitTiles;
+    const int64_t nvt = (int64_t)vtiles.size() - vt_first;
+    const int64_t nunits = (nvt + kMaxUnitTiles - 1) / kMaxUnitTiles;
     for (int64_t c = 0; c < nunits; ++c) {
-      const int64_t t0 = c * kMaxUnitTiles, t1 = std::min(nt, t0 + kMaxUnitTiles);
-      DUnit u;
+      const int64_t t0 = c * kMaxUnitTiles, t1 = std::min(nvt, t0 + kMaxUnitTiles);
+      DUnit u{};
       u.q0 = (int32_t)q0;
       u.nrows = (int32_t)nrows;
-      u.tile0 = (int32_t)(tile_base + t0);
-      u.ntiles = (int32_t)(t1 - t0);
-      u.dc0 = (int32_t)(dc0 + t0 * TW);
-      u.ncols = (int32_t)(std::min(nd, t1 * TW) - t0 * TW);
+      u.vt0 = (int32_t)(vt_first + t0);
+      u.nvt = (int32_t)(t1 - t0);
       u.split = nunits > 1 ? (int32_t)(n_dslots + c) : -1;
-      u.pad = 0;
       units.push_back(u);
       if (nunits > 1) dsplit.push_back(make_int2((int)n_dslots, (int)nunits));
     }
     if (nunits > 1) n_dslots += nunits;
   }
+  pad4();
   P.n_units = (int64_t)units.size();
   P.max_dense_per_panel = maxd;
   P.tile_cols = TW;
+  P.trp_stride = TS;
   P.panel_rows = PR;
   P.n_dslots = n_dslots;
   P.dscratch.release();
   P.dscratch_k = 0;
   SR_TRY(P.units.upload(units, s));
+  SR_TRY(P.vtiles.upload(vtiles, s));
   SR_TRY(P.dense_cols.upload(T.dense_cols, s));
   SR_TRY(P.trp.upload(trp, s));
   SR_TRY(P.d_ent.upload(de, s));
@@ -306,9 +341,9 @@ int build_exec_plan(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s) {
   sparse_traffic(ib, n_nonzero, (int64_t)ib.items.size() - n_nonzero, se, A.N, tm);
   {
     std::vector<uint8_t> seen((size_t)A.N, 0);
-    for (const DUnit& d : units) {
+    for (const VTile& d : vtiles) {
       tm.dense_col_loads += d.ncols;
-      for (int32_t k = d.dc0; k < d.dc0 + d.ncols; ++k)
+      for (int32_t k = d.col0; k < d.col0 + d.ncols; ++k)
         if (!seen[T.dense_cols[k]]) {
           seen[T.dense_cols[k]] = 1;
           ++tm.dense_distinct_cols;

@@ -236,75 +236,120 @@ __global__ void __launch_bounds__(256) sddmm_sparse_kernel(
 }
 
 // ------------------------------------------------------------------ phase D
-// Work unit = up to kMaxUnitTiles consecutive tiles of one panel (DUnit).  Entries are
-// stored tile-major: tile t, panel row r -> ent[trp[t·(P+1)+r] .. trp[t·(P+1)+r+1]) with
-// the slot relative to the tile.  A dedicated producer warp streams the unit's tiles
-// through an NST-stage shared-memory ring with cp.async.bulk (one 16-byte-aligned copy of
-// KC columns per dense column) and full/empty mbarriers, so consumer warps never meet at
-// a CTA barrier.  Consumer warp w owns the contiguous panel rows [w·RPW, (w+1)·RPW): its
-// entries of one tile are contiguous, so one coalesced load brings them in.
+// Work unit = up to kMaxUnitTiles virtual tiles of one panel (DUnit / VTile).  A dedicated
+// producer warp streams each tile through a 2- or 3-deep shared-memory ring with
+// cp.async.bulk (TMA bulk copies, SASS UBLKCP): the tile's B/Y rows (one 16-byte-aligned
+// copy of the staged columns per dense column), its panel-row offsets (trp) and its entry
+// block (and the SDDMM output indices), all completing on one full mbarrier with a
+// transaction count.  Consumer warps release a stage through an empty mbarrier, so they
+// never meet at a CTA barrier, and every load in their inner loop hits shared memory.
+// Consumer warp w owns the contiguous panel rows [w·RPW, (w+1)·RPW).
 constexpr int kDenseWarps = 8;  // consumer warps per phase-D CTA (+1 producer warp)
-constexpr int kStages = 3;
+constexpr int kMaxStages = 3;  // SpMM runs 3 stages, SDDMM 2 (its stages also carry output indices)
+constexpr int kSpmmStages = 3;
+constexpr int kSddmmStages = 2;
+constexpr size_t kUnitColsBytes = (size_t)kMaxUnitTiles * kMaxExecTile * 4;
 
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
-// Producer warp: issue stage `st` with tile tt of pass k0.
-__device__ __forceinline__ void produce_tile(float* dst, const int32_t* __restrict__ cols, int ns, int KC,
-                                             int kw, const float* __restrict__ src, int64_t ld, int k0,
-                                             uint64_t* bar, int lane) {
-  if (lane == 0) mbar_expect_tx(bar, (uint32_t)(ns * kw * 4));
-  __syncwarp();
-  for (int j = lane; j < ns; j += 32)
-    bulk_g2s(dst + (size_t)j * KC, src + (int64_t)cols[j] * ld + k0, (uint32_t)(kw * 4), bar);
-}
+struct StageLayout {
+  int b_floats;   // TW × KCP
+  int trp_ints;   // TS
+  bool oidx;
+  int nst;        // pipeline depth (<= kMaxStages)
+  __host__ __device__ size_t trp_off() const { return (size_t)b_floats * 4; }
+  __host__ __device__ size_t ent_off() const { return trp_off() + (size_t)trp_ints * 4; }
+  __host__ __device__ size_t oidx_off() const { return ent_off() + (size_t)kMaxTileEntries * 8; }
+  __host__ __device__ size_t bytes() const { return oidx_off() + (oidx ? (size_t)kMaxTileEntries * 4 : 0); }
+};
 
-// Consumer-side iteration over the unit's (pass, tile) sequence.  Calls body(tile_smem,
-// tile_index, k0, kw) for every tile, and pass_end(k0) after the last tile of a pass.
-template <int VEC, bool kBulk, typename Body, typename PassEnd>
-__device__ __forceinline__ void dense_pipeline(const DUnit& u, const int32_t* __restrict__ dense_cols,
-                                               const float* __restrict__ src, int64_t ld, int K, int KC,
-                                               int TW, float* smem, uint64_t* full, uint64_t* empty,
-                                               Body body, PassEnd pass_end) {
+template <bool kBulk, typename Body, typename PassEnd>
+__device__ __forceinline__ void dense_pipeline(const DUnit& u, const VTile* __restrict__ vtiles,
+                                               const int32_t* __restrict__ dense_cols,
+                                               const int32_t* __restrict__ trp, const int2* __restrict__ ent,
+                                               const int32_t* __restrict__ oidx, const float* __restrict__ src,
+                                               int64_t ld, int K, int KCP, const StageLayout L, char* smem,
+                                               uint64_t* full, uint64_t* empty, Body body, PassEnd pass_end) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int npass = (K + KC - 1) / KC;
-  const int total = npass * u.ntiles;
+  const int npass = (K + KCP - 1) / KCP;
+  const int total = npass * u.nvt;
+  const size_t SB = L.bytes();
   if constexpr (kBulk) {
-    if (warp == kDenseWarps) {  // producer
+    if (warp == kDenseWarps) {  // producer warp
+      // the unit's tile descriptors (lane i holds tile i) and its dense column ids (contiguous
+      // range, <= kMaxUnitTiles·kMaxExecTile) are fetched once, so issuing a tile needs no
+      // dependent global load
+      const VTile mine = lane < u.nvt ? vtiles[u.vt0 + lane] : VTile{0, 0, 0, 0};
+      const int col_lo = __shfl_sync(FULL, mine.col0, 0);
+      const VTile lastv = vtiles[u.vt0 + u.nvt - 1];
+      const int ncol_unit = lastv.col0 + lastv.ncols - col_lo;
+      const int NST = L.nst;
+      int32_t* ucols = reinterpret_cast<int32_t*>(smem + NST * SB);
+      for (int j = lane; j < ncol_unit; j += 32) ucols[j] = dense_cols[col_lo + j];
+      __syncwarp();
       for (int idx = 0; idx < total; ++idx) {
-        const int st = idx % kStages;
-        if (idx >= kStages) mbar_wait(&empty[st], ((idx - kStages) / kStages) & 1);
-        const int pass = idx / u.ntiles, tt = idx % u.ntiles;
-        const int k0 = pass * KC, kw = min(KC, K - k0), s0 = tt * TW;
-        produce_tile(smem + (size_t)st * TW * KC, dense_cols + u.dc0 + s0, min(TW, u.ncols - s0), KC, kw,
-                     src, ld, k0, &full[st], lane);
+        const int st = idx % NST;
+        if (idx >= NST) mbar_wait(&empty[st], ((idx - NST) / NST) & 1);
+        const int pass = idx / u.nvt, ti = idx % u.nvt, vt = u.vt0 + ti;
+        const int k0 = pass * KCP, kw = min(KCP, K - k0);
+        VTile v;
+        v.ent0 = __shfl_sync(FULL, mine.ent0, ti);
+        v.nent = __shfl_sync(FULL, mine.nent, ti);
+        v.col0 = __shfl_sync(FULL, mine.col0, ti);
+        v.ncols = __shfl_sync(FULL, mine.ncols, ti);
+        char* base = smem + st * SB;
+        const uint32_t bytes = (uint32_t)(v.ncols * kw * 4 + L.trp_ints * 4 + v.nent * 8 + (L.oidx ? v.nent * 4 : 0));
+        if (lane == 0) mbar_expect_tx(&full[st], bytes);
+        __syncwarp();
+        const int32_t* cols = ucols + (v.col0 - col_lo);
+        for (int j = lane; j < v.ncols; j += 32)
+          bulk_g2s(base + (size_t)j * KCP * 4, src + (int64_t)cols[j] * ld + k0, (uint32_t)(kw * 4), &full[st]);
+        if (lane == 0) bulk_g2s(base + L.trp_off(), trp + (int64_t)vt * L.trp_ints, (uint32_t)(L.trp_ints * 4),
+                                &full[st]);
+        if (lane == 1 && v.nent > 0) bulk_g2s(base + L.ent_off(), ent + v.ent0, (uint32_t)(v.nent * 8), &full[st]);
+        if (lane == 2 && L.oidx && v.nent > 0)
+          bulk_g2s(base + L.oidx_off(), oidx + v.ent0, (uint32_t)(v.nent * 4), &full[st]);
       }
       return;
     }
     for (int idx = 0; idx < total; ++idx) {
-      const int st = idx % kStages;
-      mbar_wait(&full[st], (idx / kStages) & 1);
-      const int pass = idx / u.ntiles, tt = idx % u.ntiles;
-      const int k0 = pass * KC;
-      body(smem + (size_t)st * TW * KC, u.tile0 + tt, k0, min(KC, K - k0));
+      const int st = idx % L.nst;
+      mbar_wait(&full[st], (idx / L.nst) & 1);
+      const int pass = idx / u.nvt;
+      const int k0 = pass * KCP;
+      const char* base = smem + st * SB;
+      body(reinterpret_cast<const float*>(base), reinterpret_cast<const int32_t*>(base + L.trp_off()),
+           reinterpret_cast<const int2*>(base + L.ent_off()), reinterpret_cast<const int32_t*>(base + L.oidx_off()),
+           k0, min(KCP, K - k0));
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[st]);
-      if (tt == u.ntiles - 1) pass_end(k0);
+      if (idx % u.nvt == u.nvt - 1) pass_end(k0);
     }
   } else {
     for (int idx = 0; idx < total; ++idx) {
-      const int pass = idx / u.ntiles, tt = idx % u.ntiles;
-      const int k0 = pass * KC, kw = min(KC, K - k0), s0 = tt * TW, ns = min(TW, u.ncols - s0);
+      const int pass = idx / u.nvt, vt = u.vt0 + idx % u.nvt;
+      const int k0 = pass * KCP, kw = min(KCP, K - k0);
+      const VTile v = vtiles[vt];
+      float* Bs = reinterpret_cast<float*>(smem);
+      int32_t* Ts = reinterpret_cast<int32_t*>(smem + L.trp_off());
+      int2* Es = reinterpret_cast<int2*>(smem + L.ent_off());
+      int32_t* Os = reinterpret_cast<int32_t*>(smem + L.oidx_off());
       __syncthreads();
-      for (int i = threadIdx.x; i < ns * kw; i += blockDim.x) {
+      for (int i = threadIdx.x; i < v.ncols * kw; i += blockDim.x) {
         const int j = i / kw, k = i % kw;
-        smem[(size_t)j * KC + k] = __ldg(src + (int64_t)dense_cols[u.dc0 + s0 + j] * ld + k0 + k);
+        Bs[(size_t)j * KCP + k] = __ldg(src + (int64_t)dense_cols[v.col0 + j] * ld + k0 + k);
+      }
+      for (int i = threadIdx.x; i < L.trp_ints; i += blockDim.x) Ts[i] = trp[(int64_t)vt * L.trp_ints + i];
+      for (int i = threadIdx.x; i < v.nent; i += blockDim.x) {
+        Es[i] = ent[v.ent0 + i];
+        if (L.oidx) Os[i] = oidx[v.ent0 + i];
       }
       __syncthreads();
       if (warp < kDenseWarps) {
-        body(smem, u.tile0 + tt, k0, kw);
-        if (tt == u.ntiles - 1) pass_end(k0);
+        body(Bs, Ts, Es, Os, k0, kw);
+        if (idx % u.nvt == u.nvt - 1) pass_end(k0);
       }
     }
   }
@@ -312,7 +357,7 @@ __device__ __forceinline__ void dense_pipeline(const DUnit& u, const int32_t* __
 
 __device__ __forceinline__ void dense_init_barriers(uint64_t* full, uint64_t* empty) {
   if (threadIdx.x == 0) {
-    for (int s = 0; s < kStages; ++s) {
+    for (int s = 0; s < kMaxStages; ++s) {
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], kDenseWarps);
     }
@@ -324,14 +369,15 @@ __device__ __forceinline__ void dense_init_barriers(uint64_t* full, uint64_t* em
 // SpMM dense tiles.
 template <int LPG, int VEC, int U, int RPW, bool kBulk>
 __global__ void __launch_bounds__((kDenseWarps + 1) * 32, 2) spmm_dense_kernel(
-    const DUnit* __restrict__ units, const int32_t* __restrict__ dense_cols, const int32_t* __restrict__ trp,
-    const int2* __restrict__ ent, const int32_t* __restrict__ drow_ptr, const int32_t* __restrict__ pos_out,
-    const float* __restrict__ B, int64_t ldb, float* __restrict__ C, int64_t ldc, int K, int TW, int P,
-    float* __restrict__ scratch, const int2* __restrict__ split_info, int* __restrict__ split_counter) {
+    const DUnit* __restrict__ units, const VTile* __restrict__ vtiles, const int32_t* __restrict__ dense_cols,
+    const int32_t* __restrict__ trp, const int2* __restrict__ ent, const int32_t* __restrict__ drow_ptr,
+    const int32_t* __restrict__ pos_out, const float* __restrict__ B, int64_t ldb, float* __restrict__ C,
+    int64_t ldc, int K, int TW, int TS, int P, float* __restrict__ scratch, const int2* __restrict__ split_info,
+    int* __restrict__ split_counter) {
   constexpr int G = 32 / LPG;
   constexpr int KC = LPG * VEC;
-  extern __shared__ __align__(128) float smem[];
-  __shared__ uint64_t full[kStages], empty[kStages];
+  extern __shared__ __align__(128) char smem[];
+  __shared__ uint64_t full[kMaxStages], empty[kMaxStages];
   const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
   const int warp = threadIdx.x >> 5;
   const DUnit u = units[blockIdx.x];
@@ -340,20 +386,16 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, 2) spmm_dense_kernel(
   Frag<VEC> acc[RPW];
 #pragma unroll
   for (int i = 0; i < RPW; ++i) acc[i].zero();
-  auto body = [&](const float* tile, int t, int k0, int kw) {
+  auto body = [&](const float* tile, const int32_t* rp, const int2* es, const int32_t*, int k0, int kw) {
     if (r0 >= u.nrows) return;
-    const int kk = k0 + lg * VEC;
     const bool kv = lg * VEC < kw;
-    const int32_t* rp = trp + (int64_t)t * (P + 1) + r0;
-    const int bnd = lane <= RPW ? __ldg(rp + lane) : 0;  // row bounds of this warp's rows
+    const int bnd = lane <= RPW ? rp[r0 + lane] : 0;  // row bounds of this warp's rows
     const int e_lo = __shfl_sync(FULL, bnd, 0), e_hi = __shfl_sync(FULL, bnd, RPW);
-    (void)kk;
     for (int e = e_lo; e < e_hi; e += 32) {
       const int n = min(32, e_hi - e);
-      const int2 my = lane < n ? __ldcs(ent + e + lane) : make_int2(0, 0);
+      const int2 my = lane < n ? es[e + lane] : make_int2(0, 0);
 #pragma unroll
       for (int i = 0; i < RPW; ++i) {
-        // entries of row r0+i inside this 32-entry chunk: [a, b) in lane space
         const int a = max(0, __shfl_sync(FULL, bnd, i) - e), b = min(n, __shfl_sync(FULL, bnd, i + 1) - e);
         for (int base = a; base < b; base += G * U) {
           Frag<VEC> bv[U];
@@ -390,10 +432,12 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, 2) spmm_dense_kernel(
       acc[i].zero();
     }
   };
-  dense_pipeline<VEC, kBulk>(u, dense_cols, B, ldb, K, KC, TW, smem, full, empty, body, pass_end);
+  const StageLayout L{TW * KC, TS, false, kSpmmStages};
+  dense_pipeline<kBulk>(u, vtiles, dense_cols, trp, ent, nullptr, B, ldb, K, KC, L, smem, full, empty, body,
+                        pass_end);
   if (u.split >= 0) {
     // giant panel split over several units: the last unit to finish sums the chunk
-    // partials in chunk order (deterministic) and writes the panel's dense rows
+    // partials in unit order (deterministic) and writes the panel's dense rows
     __shared__ int last;
     __threadfence();
     __syncthreads();
@@ -419,47 +463,44 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, 2) spmm_dense_kernel(
   }
 }
 
-// SDDMM dense tiles: per K pass, X fragments of the warp's rows stay in registers and every
-// tile nnz gets one dot product from shared memory; passes after the first accumulate into
-// out (same lane, same order: deterministic).
-template <int LPG, int VEC, int U, int RPW, bool kBulk>
+// SDDMM dense tiles.  Lane geometry as phase S: LPG lanes × NCH chunks of LPG·VEC columns
+// cover one nnz (K=128: 8 lanes × 4 float4, 4 nnz per warp step, 3-step shuffle reduction).
+// X fragments of the current row come from global memory (L1-resident across the tiles);
+// passes after the first (K > 256) accumulate into out (same lane, same order).
+template <int LPG, int VEC, int U, int NCH, int RPW, bool kBulk>
 __global__ void __launch_bounds__((kDenseWarps + 1) * 32, 2) sddmm_dense_kernel(
-    const DUnit* __restrict__ units, const int32_t* __restrict__ dense_cols, const int32_t* __restrict__ trp,
-    const int2* __restrict__ ent, const int32_t* __restrict__ d_oidx, const int32_t* __restrict__ pos_xrow,
-    const float* __restrict__ X, int64_t ldx, const float* __restrict__ Y, int64_t ldy, int K, int TW, int P,
-    float* __restrict__ out) {
+    const DUnit* __restrict__ units, const VTile* __restrict__ vtiles, const int32_t* __restrict__ dense_cols,
+    const int32_t* __restrict__ trp, const int2* __restrict__ ent, const int32_t* __restrict__ d_oidx,
+    const int32_t* __restrict__ pos_xrow, const float* __restrict__ X, int64_t ldx, const float* __restrict__ Y,
+    int64_t ldy, int K, int TW, int TS, float* __restrict__ out) {
   constexpr int G = 32 / LPG;
-  constexpr int KC = LPG * VEC;
-  extern __shared__ __align__(128) float smem[];
-  __shared__ uint64_t full[kStages], empty[kStages];
+  constexpr int KC = LPG * VEC;   // columns of one chunk
+  constexpr int KCP = NCH * KC;   // columns staged per pass (slot stride)
+  extern __shared__ __align__(128) char smem[];
+  __shared__ uint64_t full[kMaxStages], empty[kMaxStages];
   const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
   const int warp = threadIdx.x >> 5;
   const DUnit u = units[blockIdx.x];
   dense_init_barriers(full, empty);
   const int r0 = warp * RPW;
-  Frag<VEC> x[RPW];
-  int xk0 = -1;
-  auto body = [&](const float* tile, int t, int k0, int kw) {
+  auto body = [&](const float* tile, const int32_t* rp, const int2* es, const int32_t* os, int k0, int kw) {
     if (r0 >= u.nrows) return;
-    const bool kv = lg * VEC < kw;
-    if (k0 != xk0) {  // new K pass: this warp's X fragments
-#pragma unroll
-      for (int i = 0; i < RPW; ++i) {
-        if (r0 + i < u.nrows && kv) x[i].load_g(X + (int64_t)pos_xrow[u.q0 + r0 + i] * ldx + k0 + lg * VEC);
-        else x[i].zero();
-      }
-      xk0 = k0;
-    }
-    const int32_t* rp = trp + (int64_t)t * (P + 1) + r0;
-    const int bnd = lane <= RPW ? __ldg(rp + lane) : 0;
+    const int bnd = lane <= RPW ? rp[r0 + lane] : 0;
     const int e_lo = __shfl_sync(FULL, bnd, 0), e_hi = __shfl_sync(FULL, bnd, RPW);
     for (int e = e_lo; e < e_hi; e += 32) {
       const int n = min(32, e_hi - e);
-      const int2 my = lane < n ? __ldcs(ent + e + lane) : make_int2(0, 0);
-      const int myo = lane < n ? __ldcs(d_oidx + e + lane) : 0;
-#pragma unroll
+      const int2 my = lane < n ? es[e + lane] : make_int2(0, 0);
+      const int myo = lane < n ? os[e + lane] : 0;
+#pragma unroll 1
       for (int i = 0; i < RPW; ++i) {
         const int a = max(0, __shfl_sync(FULL, bnd, i) - e), b = min(n, __shfl_sync(FULL, bnd, i + 1) - e);
+        if (a >= b) continue;
+        Frag<VEC> x[NCH];
+        const float* xr = X + (int64_t)pos_xrow[u.q0 + r0 + i] * ldx + k0;
+#pragma unroll
+        for (int c = 0; c < NCH; ++c) {
+          if (c * KC + lg * VEC < kw) x[c].load_g(xr + c * KC + lg * VEC); else x[c].zero();
+        }
         for (int base = a; base < b; base += G * U) {
           float part[U];
 #pragma unroll
@@ -467,10 +508,15 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, 2) sddmm_dense_kernel(
             const int j = base + uu * G + g;
             const int slot = __shfl_sync(FULL, my.x, j & 31);
             float d = 0.f;
-            if (j < b && kv) {
-              Frag<VEC> y;
-              y.load_s(tile + (size_t)slot * KC + lg * VEC);
-              d = x[i].dot(y);
+            if (j < b) {
+#pragma unroll
+              for (int c = 0; c < NCH; ++c) {
+                if (c * KC + lg * VEC < kw) {
+                  Frag<VEC> y;
+                  y.load_s(tile + (size_t)slot * KCP + c * KC + lg * VEC);
+                  d += x[c].dot(y);
+                }
+              }
             }
             part[uu] = d;
           }
@@ -495,7 +541,9 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, 2) sddmm_dense_kernel(
     }
   };
   auto pass_end = [&](int) {};
-  dense_pipeline<VEC, kBulk>(u, dense_cols, Y, ldy, K, KC, TW, smem, full, empty, body, pass_end);
+  const StageLayout L{TW * KCP, TS, true, kSddmmStages};
+  dense_pipeline<kBulk>(u, vtiles, dense_cols, trp, ent, d_oidx, Y, ldy, K, KCP, L, smem, full, empty, body,
+                        pass_end);
 }
 
 // ------------------------------------------------------------------ host dispatch
@@ -516,7 +564,7 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
   constexpr int UD = 4;                   // shared-memory reads in flight per lane (phase D)
   if (P.n_units > 0) {
     const int TW = P.tile_cols;
-    const size_t smem = (size_t)kStages * TW * KC * sizeof(float);
+    const size_t smem = (size_t)kSpmmStages * StageLayout{TW * KC, P.trp_stride, false, kSpmmStages}.bytes() + kUnitColsBytes;
     if (P.n_dslots > 0 && P.dscratch_k < K) {
       SR_TRY(P.dscratch.alloc((size_t)P.n_dslots * P.panel_rows * K));
       P.dscratch_k = K;
@@ -524,8 +572,8 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
     auto launch = [&](auto kern) -> int {
       SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
       kern<<<(unsigned)P.n_units, (kDenseWarps + 1) * 32, smem, s>>>(
-          P.units.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.drow_ptr.p, P.pos_out.p, B, ldb, C, ldc, (int)K, TW,
-          P.panel_rows, P.dscratch.p, P.dsplit_info.p, P.dsplit_counter.p);
+          P.units.p, P.vtiles.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.drow_ptr.p, P.pos_out.p, B, ldb, C, ldc,
+          (int)K, TW, P.trp_stride, P.panel_rows, P.dscratch.p, P.dsplit_info.p, P.dsplit_counter.p);
       SR_CUDA_TRY(cudaGetLastError());
       return SR_OK;
     };
@@ -562,24 +610,25 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
   DevPlan& P = h->plan;
   constexpr int KC = LPG * VEC;
   constexpr int U = (LPG == 32) ? 4 : 2;
+  constexpr int NCH_D = (LPG == 32) ? 1 : NCH;  // dense: whole K per pass unless K > 256
   if (P.n_units > 0) {
     const int TW = P.tile_cols;
-    const size_t smem = (size_t)kStages * TW * KC * sizeof(float);
+    const size_t smem = (size_t)kSddmmStages * StageLayout{TW * NCH_D * KC, P.trp_stride, true, kSddmmStages}.bytes() + kUnitColsBytes;
     auto launch = [&](auto kern) -> int {
       SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
       kern<<<(unsigned)P.n_units, (kDenseWarps + 1) * 32, smem, s>>>(
-          P.units.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.d_oidx.p, P.pos_xrow.p, X, ldx, Y, ldy, (int)K, TW,
-          P.panel_rows, out);
+          P.units.p, P.vtiles.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.d_oidx.p, P.pos_xrow.p, X, ldx, Y, ldy,
+          (int)K, TW, P.trp_stride, out);
       SR_CUDA_TRY(cudaGetLastError());
       return SR_OK;
     };
     constexpr int UD = 4;
     if (P.profiling) SR_TRY(prof_begin(P, 3, s));
     if (VEC == 4) {
-      if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, 8, true>));
-      else SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, 16, true>));
+      if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 8, true>));
+      else SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 16, true>));
     } else {
-      SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, 16, false>));
+      SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 16, false>));
     }
     if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;
@@ -647,10 +696,16 @@ int launch_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64
   }
 #define SR_D(L, V, N) return run_sddmm<L, V, N>(h, X, ldx, Y, ldy, K, out, s, launches)
   if (vec) {
-    if (lpg < 32) {
-      switch (lpg) { case 1: SR_D(1, 4, 1); case 2: SR_D(2, 4, 1); case 4: SR_D(4, 4, 1); case 8: SR_D(8, 4, 1); default: SR_D(16, 4, 1); }
+    if (K <= 32) {
+      switch (lpg) { case 1: SR_D(1, 4, 1); case 2: SR_D(2, 4, 1); case 4: SR_D(4, 4, 1); default: SR_D(8, 4, 1); }
     }
-    switch (nch) { case 1: SR_D(32, 4, 1); case 2: SR_D(32, 4, 2); case 3: case 4: SR_D(32, 4, 4); default: SR_D(32, 4, 8); }
+    if (K <= 256) {  // 8 lanes x NCH float4 per nnz: 4 nnz per warp step, 3-step reductions
+      const int64_t n8 = (K + 31) / 32;
+      if (n8 <= 2) SR_D(8, 4, 2);
+      if (n8 <= 4) SR_D(8, 4, 4);
+      SR_D(8, 4, 8);
+    }
+    switch (nch) { case 3: case 4: SR_D(32, 4, 4); default: SR_D(32, 4, 8); }
   } else {
     if (lpg < 32) {
       switch (lpg) { case 1: SR_D(1, 1, 1); case 2: SR_D(2, 1, 1); case 4: SR_D(4, 1, 1); case 8: SR_D(8, 1, 1); default: SR_D(16, 1, 1); }

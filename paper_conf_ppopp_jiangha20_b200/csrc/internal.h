@@ -103,16 +103,24 @@ constexpr uint32_t kItemRMW = 1u << 31;    // C[out] += partial (row also has de
 constexpr uint32_t kItemSplit = 1u << 30;  // partial of a split long row -> scratch slot
 constexpr uint32_t kItemSlotMask = (1u << 30) - 1;
 
-// Phase-D work unit (one CTA): up to kMaxUnitTiles consecutive tiles of one panel.
+// Phase-D execution tile: <= kMaxExecTile dense columns of one panel and (a row subset of)
+// their entries; its entry block is 16-byte aligned so one bulk copy stages it.
+struct __align__(16) VTile {
+  int32_t ent0;   // first entry in d_ent / d_oidx (multiple of 4)
+  int32_t nent;   // entries in the block, padded to a multiple of 4
+  int32_t col0;   // dense_cols index of the first staged column
+  int32_t ncols;  // staged columns
+};
+// Phase-D work unit (one CTA): up to kMaxUnitTiles consecutive virtual tiles of one panel.
 struct __align__(16) DUnit {
-  int32_t q0, nrows;      // panel positions [q0, q0+nrows)
-  int32_t tile0, ntiles;  // global tile ids [tile0, tile0+ntiles)
-  int32_t dc0, ncols;     // dense_cols[dc0, dc0+ncols): the columns staged by this unit
-  int32_t split;          // -1: the unit covers its whole panel; else its partial-sum slot
-  int32_t pad;
+  int32_t q0, nrows;  // panel positions [q0, q0+nrows)
+  int32_t vt0, nvt;   // virtual tiles [vt0, vt0+nvt)
+  int32_t split;      // -1: the unit covers its whole panel; else its partial-sum slot
+  int32_t pad0, pad1, pad2;
 };
 constexpr int kMaxUnitTiles = 16;
 constexpr int kMaxExecTile = 64;
+constexpr int kMaxTileEntries = 512;
 
 // Device-resident execution plan.
 struct DevPlan {
@@ -120,7 +128,9 @@ struct DevPlan {
   DevBuf<DUnit> units;
   int64_t n_units = 0;
   DevBuf<int32_t> dense_cols;
-  DevBuf<int32_t> trp;        // per tile: panel_rows+1 offsets into d_ent (tile-major layout)
+  DevBuf<VTile> vtiles;
+  DevBuf<int32_t> trp;        // per virtual tile: trp_stride offsets relative to its entry block
+  int32_t trp_stride = 68;
   DevBuf<int32_t> drow_ptr;   // positions -> dense nnz offsets (only "row has dense nnz" is used)
   DevBuf<int2> d_ent;         // tile-major {slot in tile, __float_as_int(val)}
   DevBuf<int32_t> d_oidx;     // SDDMM output index per dense nnz (tile-major)
