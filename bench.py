@@ -49,6 +49,7 @@ def parse():
     ap.add_argument("--panel-rows", type=int, default=64)
     ap.add_argument("--tile-cols", type=int, default=64)
     ap.add_argument("--max-bucket", type=int, default=32)
+    ap.add_argument("--dense-min", type=int, default=2)
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target CPU work of cpu_baseline")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -218,7 +219,7 @@ def run_ours(args, A, ops, rank, world, local_rank):
     K = args.K
     mode = {"auto": sr.AUTO, "force": sr.FORCE, "off": sr.OFF}[args.mode]
     params = sr.default_params(mode=mode, panel_rows=args.panel_rows, tile_cols=args.tile_cols,
-                               max_bucket=args.max_bucket, world=world, rank=rank)
+                               max_bucket=args.max_bucket, dense_min=args.dense_min, world=world, rank=rank)
     M = sr.SparseMatrix.from_csr(A, device=local_rank)
     t0 = time.perf_counter()
     st = M.reorder(params)
@@ -374,7 +375,7 @@ def run_ours(args, A, ops, rank, world, local_rank):
                        "parallelism": f"row-panel shards x{world}" if world > 1 else "single GPU",
                        "l2": "512 MB write between steps (outside timed intervals); B/X/Y > L2",
                        "plan": {"mode": args.mode, "panel_rows": args.panel_rows, "tile_cols": args.tile_cols,
-                                "max_bucket": args.max_bucket, "siglen": 128, "bsize": 2, "threshold_size": 256,
+                                "max_bucket": args.max_bucket, "dense_min": args.dense_min, "siglen": 128, "bsize": 2, "threshold_size": 256,
                                 "seed": 4}},
             "roofline": roofline,
             "cpu_baseline": cpu,

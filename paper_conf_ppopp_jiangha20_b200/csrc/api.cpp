@@ -306,6 +306,9 @@ int build_exec_plan(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s) {
     for (int64_t q = 0; q < M; ++q) pout[q] = sharded ? (int32_t)(q - q0s) : perm1[q];
     SR_TRY(P.pos_xrow.upload(perm1, s));
     SR_TRY(P.pos_out.upload(pout, s));
+    std::vector<int32_t> dout((size_t)M);
+    for (int64_t q = 0; q < M; ++q) dout[q] = T.drow_ptr[q + 1] > T.drow_ptr[q] ? pout[q] : -1;
+    SR_TRY(P.dense_out.upload(dout, s));
   }
   // phase S: remainder rows in perm2 order (restricted to the shard), then zero rows
   std::vector<int2> se;

@@ -92,8 +92,8 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 }
 
 // ------------------------------------------------------------------ phase S: SpMM
-template <int LPG, int VEC, int U>
-__global__ void __launch_bounds__(256, 4) spmm_sparse_kernel(
+template <int LPG, int VEC, int U, int MINB = 4>
+__global__ void __launch_bounds__(256, MINB) spmm_sparse_kernel(
     const Item* __restrict__ items, const uint32_t* __restrict__ meta, int64_t n_items,
     const int2* __restrict__ ent, const float* __restrict__ B, int64_t ldb, float* __restrict__ C,
     int64_t ldc, int K, float* __restrict__ scratch, const int2* __restrict__ split_info,
@@ -236,122 +236,136 @@ __global__ void __launch_bounds__(256) sddmm_sparse_kernel(
 }
 
 // ------------------------------------------------------------------ phase D
-// Work unit = up to kMaxUnitTiles virtual tiles of one panel (DUnit / VTile).  A dedicated
-// producer warp streams each tile through a 2- or 3-deep shared-memory ring with
-// cp.async.bulk (TMA bulk copies, SASS UBLKCP): the tile's B/Y rows (one 16-byte-aligned
-// copy of the staged columns per dense column), its panel-row offsets (trp) and its entry
-// block (and the SDDMM output indices), all completing on one full mbarrier with a
-// transaction count.  Consumer warps release a stage through an empty mbarrier, so they
-// never meet at a CTA barrier, and every load in their inner loop hits shared memory.
+// Persistent CTAs (2 per SM) walk the work units (DUnit = up to kMaxUnitTiles virtual tiles
+// of one panel, VTile) round-robin.  A dedicated producer warp streams every tile of every
+// unit of its CTA through an NST-deep shared-memory ring: the tile's B/Y rows (one
+// cp.async.bulk per dense column, 16-byte aligned, K·4 bytes), its panel-row offsets (trp),
+// its entry block (and SDDMM output indices) and a 32-byte stage header, all completing on
+// one full mbarrier with a transaction count.  Consumer warps (8) release stages through
+// an empty mbarrier, so consumers never meet at a CTA barrier and unit boundaries cost no
+// pipeline drain: unit n+1's tiles stream in while unit n's results are stored.
 // Consumer warp w owns the contiguous panel rows [w·RPW, (w+1)·RPW).
 constexpr int kDenseWarps = 8;  // consumer warps per phase-D CTA (+1 producer warp)
-constexpr int kMaxStages = 3;  // SpMM runs 3 stages, SDDMM 2 (its stages also carry output indices)
+constexpr int kMaxStages = 3;   // SpMM runs 3 stages, SDDMM 2 (its stages also carry output indices)
 constexpr int kSpmmStages = 3;
 constexpr int kSddmmStages = 2;
+constexpr int kDenseCtasPerSM = 2;
 constexpr size_t kUnitColsBytes = (size_t)kMaxUnitTiles * kMaxExecTile * 4;
 
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
+__device__ __forceinline__ void consumers_sync() {  // named barrier over the 8 consumer warps
+  asm volatile("bar.sync 1, %0;" ::"n"(kDenseWarps * 32) : "memory");
+}
+
+// Stage header written by the producer (plain st.shared before its arrive; the arrive has
+// release semantics and the consumers' wait acquire semantics).
+struct __align__(16) StageHdr {
+  int32_t q0, nrows, split, flags;
+  int32_t k0, kw, uid, pad;
+};
+constexpr int kFirstOfPass = 1, kLastOfPass = 2, kFirstOfUnit = 4, kLastOfUnit = 8, kLastOfCta = 16;
 
 struct StageLayout {
   int b_floats;   // TW × KCP
   int trp_ints;   // TS
   bool oidx;
   int nst;        // pipeline depth (<= kMaxStages)
-  __host__ __device__ size_t trp_off() const { return (size_t)b_floats * 4; }
+  int dbg;        // measurement knobs (SR_DEBUG_DENSE): 1 = skip consumer math, 2 = skip copies
+  bool bulk;      // TMA bulk copies (16-byte-aligned rows); else the producer copies with LDG/STS
+  __host__ __device__ size_t b_off() const { return sizeof(StageHdr); }
+  __host__ __device__ size_t trp_off() const { return b_off() + (size_t)b_floats * 4; }
   __host__ __device__ size_t ent_off() const { return trp_off() + (size_t)trp_ints * 4; }
   __host__ __device__ size_t oidx_off() const { return ent_off() + (size_t)kMaxTileEntries * 8; }
   __host__ __device__ size_t bytes() const { return oidx_off() + (oidx ? (size_t)kMaxTileEntries * 4 : 0); }
+  __host__ size_t smem(int nst_) const { return (size_t)nst_ * bytes() + kUnitColsBytes; }
 };
 
-template <bool kBulk, typename Body, typename PassEnd>
-__device__ __forceinline__ void dense_pipeline(const DUnit& u, const VTile* __restrict__ vtiles,
-                                               const int32_t* __restrict__ dense_cols,
-                                               const int32_t* __restrict__ trp, const int2* __restrict__ ent,
-                                               const int32_t* __restrict__ oidx, const float* __restrict__ src,
-                                               int64_t ld, int K, int KCP, const StageLayout L, char* smem,
-                                               uint64_t* full, uint64_t* empty, Body body, PassEnd pass_end) {
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int npass = (K + KCP - 1) / KCP;
-  const int total = npass * u.nvt;
+// Producer warp: every tile of every unit of this CTA.
+__device__ __forceinline__ void dense_produce(const DUnit* __restrict__ units, int n_units,
+                                              const VTile* __restrict__ vtiles,
+                                              const int32_t* __restrict__ dense_cols,
+                                              const int32_t* __restrict__ trp, const int2* __restrict__ ent,
+                                              const int32_t* __restrict__ oidx, const float* __restrict__ src,
+                                              int64_t ld, int K, int KCP, const StageLayout& L, char* smem,
+                                              uint64_t* full, uint64_t* empty) {
+  const int lane = threadIdx.x & 31;
   const size_t SB = L.bytes();
-  if constexpr (kBulk) {
-    if (warp == kDenseWarps) {  // producer warp
-      // the unit's tile descriptors (lane i holds tile i) and its dense column ids (contiguous
-      // range, <= kMaxUnitTiles·kMaxExecTile) are fetched once, so issuing a tile needs no
-      // dependent global load
-      const VTile mine = lane < u.nvt ? vtiles[u.vt0 + lane] : VTile{0, 0, 0, 0};
-      const int col_lo = __shfl_sync(FULL, mine.col0, 0);
-      const VTile lastv = vtiles[u.vt0 + u.nvt - 1];
-      const int ncol_unit = lastv.col0 + lastv.ncols - col_lo;
-      const int NST = L.nst;
-      int32_t* ucols = reinterpret_cast<int32_t*>(smem + NST * SB);
-      for (int j = lane; j < ncol_unit; j += 32) ucols[j] = dense_cols[col_lo + j];
-      __syncwarp();
-      for (int idx = 0; idx < total; ++idx) {
-        const int st = idx % NST;
-        if (idx >= NST) mbar_wait(&empty[st], ((idx - NST) / NST) & 1);
-        const int pass = idx / u.nvt, ti = idx % u.nvt, vt = u.vt0 + ti;
-        const int k0 = pass * KCP, kw = min(KCP, K - k0);
+  int32_t* ucols = reinterpret_cast<int32_t*>(smem + L.nst * SB);
+  const int npass = (K + KCP - 1) / KCP;
+  int idx = 0;
+  for (int uid = blockIdx.x; uid < n_units; uid += gridDim.x) {
+    const DUnit u = units[uid];
+    const bool last_unit = uid + (int)gridDim.x >= n_units;
+    // the unit's tile descriptors (lane i holds tile i) and its dense column ids (contiguous,
+    // <= kMaxUnitTiles·kMaxExecTile) are fetched once per unit
+    const VTile mine = lane < u.nvt ? vtiles[u.vt0 + lane] : VTile{0, 0, 0, 0};
+    const int col_lo = __shfl_sync(FULL, mine.col0, 0);
+    const int last_col0 = __shfl_sync(FULL, mine.col0, u.nvt - 1), last_nc = __shfl_sync(FULL, mine.ncols, u.nvt - 1);
+    const int ncol_unit = last_col0 + last_nc - col_lo;
+    for (int j = lane; j < ncol_unit; j += 32) ucols[j] = dense_cols[col_lo + j];
+    __syncwarp();
+    for (int pass = 0; pass < npass; ++pass) {
+      const int k0 = pass * KCP, kw = min(KCP, K - k0);
+      for (int ti = 0; ti < u.nvt; ++ti, ++idx) {
+        const int st = idx % L.nst;
+        if (idx >= L.nst) mbar_wait(&empty[st], ((idx - L.nst) / L.nst) & 1);
         VTile v;
         v.ent0 = __shfl_sync(FULL, mine.ent0, ti);
         v.nent = __shfl_sync(FULL, mine.nent, ti);
         v.col0 = __shfl_sync(FULL, mine.col0, ti);
         v.ncols = __shfl_sync(FULL, mine.ncols, ti);
         char* base = smem + st * SB;
-        const uint32_t bytes = (uint32_t)(v.ncols * kw * 4 + L.trp_ints * 4 + v.nent * 8 + (L.oidx ? v.nent * 4 : 0));
+        if (lane == 0) {
+          StageHdr* h = reinterpret_cast<StageHdr*>(base);
+          int f = 0;
+          if (ti == 0) f |= kFirstOfPass;
+          if (ti == u.nvt - 1) f |= kLastOfPass;
+          if (ti == 0 && pass == 0) f |= kFirstOfUnit;
+          if (ti == u.nvt - 1 && pass == npass - 1) f |= kLastOfUnit | (last_unit ? kLastOfCta : 0);
+          *h = StageHdr{u.q0, u.nrows, u.split, f, k0, kw, uid, 0};
+        }
+        const int vt = u.vt0 + ti;
+        if (L.dbg & 2) {  // measurement knob: no copies
+          if (lane == 0) mbar_arrive(&full[st]);
+          continue;
+        }
+        if (!L.bulk) {  // unaligned operands (scalar path): plain loads and shared stores
+          float* bs = reinterpret_cast<float*>(base + L.b_off());
+          const int32_t* cols = ucols + (v.col0 - col_lo);
+          for (int i = lane; i < v.ncols * kw; i += 32) {
+            const int j = i / kw, k = i - j * kw;
+            bs[(size_t)j * KCP + k] = __ldg(src + (int64_t)cols[j] * ld + k0 + k);
+          }
+          int32_t* ts = reinterpret_cast<int32_t*>(base + L.trp_off());
+          for (int i = lane; i < L.trp_ints; i += 32) ts[i] = trp[(int64_t)vt * L.trp_ints + i];
+          int2* es = reinterpret_cast<int2*>(base + L.ent_off());
+          int32_t* os = reinterpret_cast<int32_t*>(base + L.oidx_off());
+          for (int i = lane; i < v.nent; i += 32) {
+            es[i] = ent[v.ent0 + i];
+            if (L.oidx) os[i] = oidx[v.ent0 + i];
+          }
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&full[st]);
+          continue;
+        }
+        const uint32_t bytes =
+            (uint32_t)(v.ncols * kw * 4 + L.trp_ints * 4 + v.nent * 8 + (L.oidx ? v.nent * 4 : 0));
         if (lane == 0) mbar_expect_tx(&full[st], bytes);
         __syncwarp();
         const int32_t* cols = ucols + (v.col0 - col_lo);
         for (int j = lane; j < v.ncols; j += 32)
-          bulk_g2s(base + (size_t)j * KCP * 4, src + (int64_t)cols[j] * ld + k0, (uint32_t)(kw * 4), &full[st]);
-        if (lane == 0) bulk_g2s(base + L.trp_off(), trp + (int64_t)vt * L.trp_ints, (uint32_t)(L.trp_ints * 4),
-                                &full[st]);
+          bulk_g2s(base + L.b_off() + (size_t)j * KCP * 4, src + (int64_t)cols[j] * ld + k0, (uint32_t)(kw * 4),
+                   &full[st]);
+        if (lane == 0)
+          bulk_g2s(base + L.trp_off(), trp + (int64_t)vt * L.trp_ints, (uint32_t)(L.trp_ints * 4), &full[st]);
         if (lane == 1 && v.nent > 0) bulk_g2s(base + L.ent_off(), ent + v.ent0, (uint32_t)(v.nent * 8), &full[st]);
         if (lane == 2 && L.oidx && v.nent > 0)
           bulk_g2s(base + L.oidx_off(), oidx + v.ent0, (uint32_t)(v.nent * 4), &full[st]);
       }
-      return;
     }
-    for (int idx = 0; idx < total; ++idx) {
-      const int st = idx % L.nst;
-      mbar_wait(&full[st], (idx / L.nst) & 1);
-      const int pass = idx / u.nvt;
-      const int k0 = pass * KCP;
-      const char* base = smem + st * SB;
-      body(reinterpret_cast<const float*>(base), reinterpret_cast<const int32_t*>(base + L.trp_off()),
-           reinterpret_cast<const int2*>(base + L.ent_off()), reinterpret_cast<const int32_t*>(base + L.oidx_off()),
-           k0, min(KCP, K - k0));
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&empty[st]);
-      if (idx % u.nvt == u.nvt - 1) pass_end(k0);
-    }
-  } else {
-    for (int idx = 0; idx < total; ++idx) {
-      const int pass = idx / u.nvt, vt = u.vt0 + idx % u.nvt;
-      const int k0 = pass * KCP, kw = min(KCP, K - k0);
-      const VTile v = vtiles[vt];
-      float* Bs = reinterpret_cast<float*>(smem);
-      int32_t* Ts = reinterpret_cast<int32_t*>(smem + L.trp_off());
-      int2* Es = reinterpret_cast<int2*>(smem + L.ent_off());
-      int32_t* Os = reinterpret_cast<int32_t*>(smem + L.oidx_off());
-      __syncthreads();
-      for (int i = threadIdx.x; i < v.ncols * kw; i += blockDim.x) {
-        const int j = i / kw, k = i % kw;
-        Bs[(size_t)j * KCP + k] = __ldg(src + (int64_t)dense_cols[v.col0 + j] * ld + k0 + k);
-      }
-      for (int i = threadIdx.x; i < L.trp_ints; i += blockDim.x) Ts[i] = trp[(int64_t)vt * L.trp_ints + i];
-      for (int i = threadIdx.x; i < v.nent; i += blockDim.x) {
-        Es[i] = ent[v.ent0 + i];
-        if (L.oidx) Os[i] = oidx[v.ent0 + i];
-      }
-      __syncthreads();
-      if (warp < kDenseWarps) {
-        body(Bs, Ts, Es, Os, k0, kw);
-        if (idx % u.nvt == u.nvt - 1) pass_end(k0);
-      }
-    }
+    __syncwarp();
   }
 }
 
@@ -367,99 +381,116 @@ __device__ __forceinline__ void dense_init_barriers(uint64_t* full, uint64_t* em
 }
 
 // SpMM dense tiles.
-template <int LPG, int VEC, int U, int RPW, bool kBulk>
-__global__ void __launch_bounds__((kDenseWarps + 1) * 32, 2) spmm_dense_kernel(
-    const DUnit* __restrict__ units, const VTile* __restrict__ vtiles, const int32_t* __restrict__ dense_cols,
-    const int32_t* __restrict__ trp, const int2* __restrict__ ent, const int32_t* __restrict__ drow_ptr,
-    const int32_t* __restrict__ pos_out, const float* __restrict__ B, int64_t ldb, float* __restrict__ C,
+template <int LPG, int VEC, int U, int RPW>
+__global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) spmm_dense_kernel(
+    const DUnit* __restrict__ units, int n_units, const VTile* __restrict__ vtiles,
+    const int32_t* __restrict__ dense_cols, const int32_t* __restrict__ trp, const int2* __restrict__ ent,
+    const int32_t* __restrict__ dense_out, const float* __restrict__ B, int64_t ldb, float* __restrict__ C,
     int64_t ldc, int K, int TW, int TS, int P, float* __restrict__ scratch, const int2* __restrict__ split_info,
-    int* __restrict__ split_counter) {
+    int* __restrict__ split_counter, int dbg) {
   constexpr int G = 32 / LPG;
   constexpr int KC = LPG * VEC;
   extern __shared__ __align__(128) char smem[];
   __shared__ uint64_t full[kMaxStages], empty[kMaxStages];
+  __shared__ int last_ticket;
   const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
   const int warp = threadIdx.x >> 5;
-  const DUnit u = units[blockIdx.x];
+  const StageLayout L{TW * KC, TS, false, kSpmmStages, dbg >> 1, (dbg & 1) != 0};
   dense_init_barriers(full, empty);
+  if (warp == kDenseWarps) {
+    dense_produce(units, n_units, vtiles, dense_cols, trp, ent, nullptr, B, ldb, K, KC, L, smem, full, empty);
+    return;
+  }
+  const size_t SB = L.bytes();
   const int r0 = warp * RPW;
   Frag<VEC> acc[RPW];
+  int out_row = -1;  // lane i < RPW: output row of panel row r0+i (-1: no dense nnz)
+  for (int idx = 0;; ++idx) {
+    const int st = idx % L.nst;
+    mbar_wait(&full[st], (idx / L.nst) & 1);
+    const char* base = smem + st * SB;
+    const StageHdr hd = *reinterpret_cast<const StageHdr*>(base);
+    if (hd.flags & kFirstOfUnit)
+      out_row = (lane < RPW && r0 + lane < hd.nrows) ? dense_out[hd.q0 + r0 + lane] : -1;
+    if (hd.flags & kFirstOfPass) {
 #pragma unroll
-  for (int i = 0; i < RPW; ++i) acc[i].zero();
-  auto body = [&](const float* tile, const int32_t* rp, const int2* es, const int32_t*, int k0, int kw) {
-    if (r0 >= u.nrows) return;
-    const bool kv = lg * VEC < kw;
-    const int bnd = lane <= RPW ? rp[r0 + lane] : 0;  // row bounds of this warp's rows
-    const int e_lo = __shfl_sync(FULL, bnd, 0), e_hi = __shfl_sync(FULL, bnd, RPW);
-    for (int e = e_lo; e < e_hi; e += 32) {
-      const int n = min(32, e_hi - e);
-      const int2 my = lane < n ? es[e + lane] : make_int2(0, 0);
+      for (int i = 0; i < RPW; ++i) acc[i].zero();
+    }
+    if (!(L.dbg & 1) && r0 < hd.nrows && lg * VEC < hd.kw) {
+      // entries and row bounds come straight from shared memory (broadcast loads): per nnz
+      // one LDS.64 of (slot, value), one LDS.128 of the staged row, four FFMA
+      const float* tcol = reinterpret_cast<const float*>(base + L.b_off()) + lg * VEC;
+      const int32_t* rp = reinterpret_cast<const int32_t*>(base + L.trp_off());
+      const int2* es = reinterpret_cast<const int2*>(base + L.ent_off());
 #pragma unroll
       for (int i = 0; i < RPW; ++i) {
-        const int a = max(0, __shfl_sync(FULL, bnd, i) - e), b = min(n, __shfl_sync(FULL, bnd, i + 1) - e);
-        for (int base = a; base < b; base += G * U) {
+        const int b0 = rp[r0 + i], b1 = rp[r0 + i + 1];
+        int e = b0 + g;
+        for (; e + (U - 1) * G < b1; e += U * G) {
+          int2 en[U];
+#pragma unroll
+          for (int uu = 0; uu < U; ++uu) en[uu] = es[e + uu * G];
           Frag<VEC> bv[U];
-          float av[U];
 #pragma unroll
-          for (int uu = 0; uu < U; ++uu) {
-            const int j = base + uu * G + g;
-            const int slot = __shfl_sync(FULL, my.x, j & 31);
-            const float v = __int_as_float(__shfl_sync(FULL, my.y, j & 31));
-            const bool ok = j < b && kv;
-            av[uu] = ok ? v : 0.f;
-            if (ok) bv[uu].load_s(tile + (size_t)slot * KC + lg * VEC); else bv[uu].zero();
+          for (int uu = 0; uu < U; ++uu) bv[uu].load_s(tcol + (size_t)en[uu].x * KC);
+#pragma unroll
+          for (int uu = 0; uu < U; ++uu) acc[i].fma(__int_as_float(en[uu].y), bv[uu]);
+        }
+        for (; e < b1; e += G) {
+          const int2 en = es[e];
+          Frag<VEC> bv;
+          bv.load_s(tcol + (size_t)en.x * KC);
+          acc[i].fma(__int_as_float(en.y), bv);
+        }
+      }
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[st]);
+    if (hd.flags & kLastOfPass) {
+      const int kk = hd.k0 + lg * VEC;
+      const bool kv = kk < K;
+#pragma unroll
+      for (int i = 0; i < RPW; ++i) {
+#pragma unroll
+        for (int off = LPG; off < 32; off <<= 1) acc[i].xor_add(off);
+        const int orow = __shfl_sync(FULL, out_row, i);
+        if (r0 + i < hd.nrows && g == 0 && kv) {
+          if (hd.split >= 0)
+            acc[i].store(scratch + ((int64_t)hd.split * P + r0 + i) * K + kk);
+          else if (orow >= 0)
+            acc[i].store_cs(C + (int64_t)orow * ldc + kk);
+        }
+      }
+    }
+    if ((hd.flags & kLastOfUnit) && hd.split >= 0) {
+      // giant panel split over several units: the last unit to finish sums the chunk
+      // partials in unit order (deterministic) and writes the panel's dense rows
+      __threadfence();
+      consumers_sync();
+      const int2 si = split_info[hd.split];
+      if (threadIdx.x == 0) last_ticket = (atomicAdd(split_counter + si.x, 1) == si.y - 1);
+      consumers_sync();
+      if (last_ticket) {
+        __threadfence();
+        for (int i = 0; i < RPW; ++i) {
+          const int orow = __shfl_sync(FULL, out_row, i);
+          if (r0 + i >= hd.nrows || orow < 0) continue;
+          for (int k = lane * VEC; k < K; k += 32 * VEC) {
+            Frag<VEC> s;
+            s.zero();
+            for (int c = 0; c < si.y; ++c) {
+              Frag<VEC> part;
+              part.load_cg(scratch + ((int64_t)(si.x + c) * P + r0 + i) * K + k);
+              s.add(part);
+            }
+            s.store_cs(C + (int64_t)orow * ldc + k);
           }
-#pragma unroll
-          for (int uu = 0; uu < U; ++uu) acc[i].fma(av[uu], bv[uu]);
         }
+        consumers_sync();
+        if (threadIdx.x == 0) split_counter[si.x] = 0;
       }
     }
-  };
-  auto pass_end = [&](int k0) {
-    const int kk = k0 + lg * VEC;
-    const bool kv = kk < K;
-#pragma unroll
-    for (int i = 0; i < RPW; ++i) {
-#pragma unroll
-      for (int off = LPG; off < 32; off <<= 1) acc[i].xor_add(off);
-      const int r = r0 + i;
-      if (r < u.nrows && g == 0 && kv) {
-        if (u.split >= 0)
-          acc[i].store(scratch + ((int64_t)u.split * P + r) * K + kk);
-        else if (drow_ptr[u.q0 + r + 1] > drow_ptr[u.q0 + r])
-          acc[i].store_cs(C + (int64_t)pos_out[u.q0 + r] * ldc + kk);
-      }
-      acc[i].zero();
-    }
-  };
-  const StageLayout L{TW * KC, TS, false, kSpmmStages};
-  dense_pipeline<kBulk>(u, vtiles, dense_cols, trp, ent, nullptr, B, ldb, K, KC, L, smem, full, empty, body,
-                        pass_end);
-  if (u.split >= 0) {
-    // giant panel split over several units: the last unit to finish sums the chunk
-    // partials in unit order (deterministic) and writes the panel's dense rows
-    __shared__ int last;
-    __threadfence();
-    __syncthreads();
-    const int2 si = split_info[u.split];
-    if (threadIdx.x == 0) last = (atomicAdd(split_counter + si.x, 1) == si.y - 1);
-    __syncthreads();
-    if (!last) return;
-    __threadfence();
-    for (int r = warp; r < u.nrows; r += kDenseWarps + 1) {
-      if (drow_ptr[u.q0 + r + 1] == drow_ptr[u.q0 + r]) continue;
-      for (int k = lane * VEC; k < K; k += 32 * VEC) {
-        Frag<VEC> s;
-        s.zero();
-        for (int c = 0; c < si.y; ++c) {
-          Frag<VEC> part;
-          part.load_cg(scratch + ((int64_t)(si.x + c) * P + r) * K + k);
-          s.add(part);
-        }
-        s.store_cs(C + (int64_t)pos_out[u.q0 + r] * ldc + k);
-      }
-    }
-    if (threadIdx.x == 0) split_counter[si.x] = 0;
+    if (hd.flags & kLastOfCta) break;
   }
 }
 
@@ -467,12 +498,13 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, 2) spmm_dense_kernel(
 // cover one nnz (K=128: 8 lanes × 4 float4, 4 nnz per warp step, 3-step shuffle reduction).
 // X fragments of the current row come from global memory (L1-resident across the tiles);
 // passes after the first (K > 256) accumulate into out (same lane, same order).
-template <int LPG, int VEC, int U, int NCH, int RPW, bool kBulk>
-__global__ void __launch_bounds__((kDenseWarps + 1) * 32, 2) sddmm_dense_kernel(
-    const DUnit* __restrict__ units, const VTile* __restrict__ vtiles, const int32_t* __restrict__ dense_cols,
-    const int32_t* __restrict__ trp, const int2* __restrict__ ent, const int32_t* __restrict__ d_oidx,
-    const int32_t* __restrict__ pos_xrow, const float* __restrict__ X, int64_t ldx, const float* __restrict__ Y,
-    int64_t ldy, int K, int TW, int TS, float* __restrict__ out) {
+template <int LPG, int VEC, int U, int NCH, int RPW>
+__global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) sddmm_dense_kernel(
+    const DUnit* __restrict__ units, int n_units, const VTile* __restrict__ vtiles,
+    const int32_t* __restrict__ dense_cols, const int32_t* __restrict__ trp, const int2* __restrict__ ent,
+    const int32_t* __restrict__ d_oidx, const int32_t* __restrict__ pos_xrow, const float* __restrict__ X,
+    int64_t ldx, const float* __restrict__ Y, int64_t ldy, int K, int TW, int TS, float* __restrict__ out,
+    int dbg) {
   constexpr int G = 32 / LPG;
   constexpr int KC = LPG * VEC;   // columns of one chunk
   constexpr int KCP = NCH * KC;   // columns staged per pass (slot stride)
@@ -480,42 +512,55 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, 2) sddmm_dense_kernel(
   __shared__ uint64_t full[kMaxStages], empty[kMaxStages];
   const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
   const int warp = threadIdx.x >> 5;
-  const DUnit u = units[blockIdx.x];
+  const StageLayout L{TW * KCP, TS, true, kSddmmStages, dbg >> 1, (dbg & 1) != 0};
   dense_init_barriers(full, empty);
+  if (warp == kDenseWarps) {
+    dense_produce(units, n_units, vtiles, dense_cols, trp, ent, d_oidx, Y, ldy, K, KCP, L, smem, full, empty);
+    return;
+  }
+  const size_t SB = L.bytes();
   const int r0 = warp * RPW;
-  auto body = [&](const float* tile, const int32_t* rp, const int2* es, const int32_t* os, int k0, int kw) {
-    if (r0 >= u.nrows) return;
-    const int bnd = lane <= RPW ? rp[r0 + lane] : 0;
-    const int e_lo = __shfl_sync(FULL, bnd, 0), e_hi = __shfl_sync(FULL, bnd, RPW);
-    for (int e = e_lo; e < e_hi; e += 32) {
-      const int n = min(32, e_hi - e);
-      const int2 my = lane < n ? es[e + lane] : make_int2(0, 0);
-      const int myo = lane < n ? os[e + lane] : 0;
+  int xrow = 0;  // lane i < RPW: X row of panel row r0+i
+  for (int idx = 0;; ++idx) {
+    const int st = idx % L.nst;
+    mbar_wait(&full[st], (idx / L.nst) & 1);
+    const char* base = smem + st * SB;
+    const StageHdr hd = *reinterpret_cast<const StageHdr*>(base);
+    if (hd.flags & kFirstOfUnit) xrow = (lane < RPW && r0 + lane < hd.nrows) ? pos_xrow[hd.q0 + r0 + lane] : 0;
+    if (!(L.dbg & 1) && r0 < hd.nrows) {
+      const float* tile = reinterpret_cast<const float*>(base + L.b_off());
+      const int32_t* rp = reinterpret_cast<const int32_t*>(base + L.trp_off());
+      const int2* es = reinterpret_cast<const int2*>(base + L.ent_off());
+      const int32_t* os = reinterpret_cast<const int32_t*>(base + L.oidx_off());
+      const int k0 = hd.k0, kw = hd.kw;
 #pragma unroll 1
       for (int i = 0; i < RPW; ++i) {
-        const int a = max(0, __shfl_sync(FULL, bnd, i) - e), b = min(n, __shfl_sync(FULL, bnd, i + 1) - e);
-        if (a >= b) continue;
+        const int b0 = rp[r0 + i], b1 = rp[r0 + i + 1];
+        const int xr_i = __shfl_sync(FULL, xrow, i);
+        if (b0 >= b1) continue;
         Frag<VEC> x[NCH];
-        const float* xr = X + (int64_t)pos_xrow[u.q0 + r0 + i] * ldx + k0;
+        const float* xr = X + (int64_t)xr_i * ldx + k0;
 #pragma unroll
         for (int c = 0; c < NCH; ++c) {
           if (c * KC + lg * VEC < kw) x[c].load_g(xr + c * KC + lg * VEC); else x[c].zero();
         }
-        for (int base = a; base < b; base += G * U) {
+        for (int bse = b0; bse < b1; bse += G * U) {
           float part[U];
+          int2 en[U];
 #pragma unroll
           for (int uu = 0; uu < U; ++uu) {
-            const int j = base + uu * G + g;
-            const int slot = __shfl_sync(FULL, my.x, j & 31);
-            float d = 0.f;
-            if (j < b) {
+            const int j = bse + uu * G + g;
+            en[uu] = j < b1 ? es[j] : make_int2(0, 0);
+          }
 #pragma unroll
-              for (int c = 0; c < NCH; ++c) {
-                if (c * KC + lg * VEC < kw) {
-                  Frag<VEC> y;
-                  y.load_s(tile + (size_t)slot * KCP + c * KC + lg * VEC);
-                  d += x[c].dot(y);
-                }
+          for (int uu = 0; uu < U; ++uu) {
+            float d = 0.f;
+#pragma unroll
+            for (int c = 0; c < NCH; ++c) {
+              if (c * KC + lg * VEC < kw) {
+                Frag<VEC> y;
+                y.load_s(tile + (size_t)en[uu].x * KCP + c * KC + lg * VEC);
+                d += x[c].dot(y);
               }
             }
             part[uu] = d;
@@ -525,25 +570,25 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, 2) sddmm_dense_kernel(
 #pragma unroll
             for (int off = LPG / 2; off > 0; off >>= 1) part[uu] += __shfl_xor_sync(FULL, part[uu], off);
           }
+          if (lg == 0) {
 #pragma unroll
-          for (int uu = 0; uu < U; ++uu) {
-            const int j = base + uu * G + g;
-            const float v = __int_as_float(__shfl_sync(FULL, my.y, j & 31));
-            const int o = __shfl_sync(FULL, myo, j & 31);
-            if (lg == 0 && j < b) {
-              float res = v * part[uu];
-              if (k0 > 0) res += out[o];
-              out[o] = res;
+            for (int uu = 0; uu < U; ++uu) {
+              const int j = bse + uu * G + g;
+              if (j < b1) {
+                const int o = os[j];
+                float res = __int_as_float(en[uu].y) * part[uu];
+                if (k0 > 0) res += out[o];
+                out[o] = res;
+              }
             }
           }
         }
       }
     }
-  };
-  auto pass_end = [&](int) {};
-  const StageLayout L{TW * KCP, TS, true, kSddmmStages};
-  dense_pipeline<kBulk>(u, vtiles, dense_cols, trp, ent, d_oidx, Y, ldy, K, KCP, L, smem, full, empty, body,
-                        pass_end);
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[st]);
+    if (hd.flags & kLastOfCta) break;
+  }
 }
 
 // ------------------------------------------------------------------ host dispatch
@@ -555,6 +600,35 @@ inline int next_pow2(int x) {
 
 constexpr int kSparseWarps = 8;
 
+// Phase-D launch knobs: SR_DEBUG_DENSE (measurement only, see StageLayout::dbg) and the
+// persistent grid (kDenseCtasPerSM CTAs per SM, never more CTAs than units).
+int dense_dbg() {
+  static const int v = [] {
+    const char* d = getenv("SR_DEBUG_DENSE");
+    return d ? (atoi(d) & 3) : 0;
+  }();
+  return v;
+}
+
+int sparse_variant() {
+  static const int v = [] {
+    const char* d = getenv("SR_SPARSE_VARIANT");
+    return d ? atoi(d) : 0;
+  }();
+  return v;
+}
+
+int num_sms() {
+  static int n = 0;
+  if (n == 0) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
+  }
+  return n;
+}
+
 template <int LPG, int VEC>
 int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int64_t ldc,
              cudaStream_t s, int32_t* launches) {
@@ -564,26 +638,24 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
   constexpr int UD = 4;                   // shared-memory reads in flight per lane (phase D)
   if (P.n_units > 0) {
     const int TW = P.tile_cols;
-    const size_t smem = (size_t)kSpmmStages * StageLayout{TW * KC, P.trp_stride, false, kSpmmStages}.bytes() + kUnitColsBytes;
+    const size_t smem = StageLayout{TW * KC, P.trp_stride, false, kSpmmStages, 0, true}.smem(kSpmmStages);
     if (P.n_dslots > 0 && P.dscratch_k < K) {
       SR_TRY(P.dscratch.alloc((size_t)P.n_dslots * P.panel_rows * K));
       P.dscratch_k = K;
     }
+    const unsigned grid = (unsigned)std::min<int64_t>(P.n_units, (int64_t)kDenseCtasPerSM * num_sms());
+    const int flags = (VEC == 4 ? 1 : 0) | (dense_dbg() << 1);
     auto launch = [&](auto kern) -> int {
       SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-      kern<<<(unsigned)P.n_units, (kDenseWarps + 1) * 32, smem, s>>>(
-          P.units.p, P.vtiles.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.drow_ptr.p, P.pos_out.p, B, ldb, C, ldc,
-          (int)K, TW, P.trp_stride, P.panel_rows, P.dscratch.p, P.dsplit_info.p, P.dsplit_counter.p);
+      kern<<<grid, (kDenseWarps + 1) * 32, smem, s>>>(
+          P.units.p, (int)P.n_units, P.vtiles.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.dense_out.p, B, ldb, C, ldc,
+          (int)K, TW, P.trp_stride, P.panel_rows, P.dscratch.p, P.dsplit_info.p, P.dsplit_counter.p, flags);
       SR_CUDA_TRY(cudaGetLastError());
       return SR_OK;
     };
     if (P.profiling) SR_TRY(prof_begin(P, 1, s));
-    if (VEC == 4) {
-      if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 8, true>));
-      else SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 16, true>));
-    } else {
-      SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 16, false>));
-    }
+    if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 8>));
+    else SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 16>));
     if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;
   }
@@ -594,9 +666,16 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
     }
     const unsigned grid = (unsigned)((P.n_items + kSparseWarps - 1) / kSparseWarps);
     if (P.profiling) SR_TRY(prof_begin(P, 2, s));
-    spmm_sparse_kernel<LPG, VEC, U><<<grid, kSparseWarps * 32, 0, s>>>(
-        P.items.p, P.item_meta.p, P.n_items, P.s_ent.p, B, ldb, C, ldc, (int)K, P.scratch.p,
-        P.split_info.p, P.split_counter.p);
+    auto go = [&](auto kern) {
+      kern<<<grid, kSparseWarps * 32, 0, s>>>(P.items.p, P.item_meta.p, P.n_items, P.s_ent.p, B, ldb, C, ldc, (int)K,
+                                               P.scratch.p, P.split_info.p, P.split_counter.p);
+    };
+    // SR_SPARSE_VARIANT (tuning knob): 0 = U 8 / 4 CTAs per SM (default), 1 = U 4 / 6, 2 = U 2 / 8
+    switch (sparse_variant()) {
+      case 1: go(spmm_sparse_kernel<LPG, VEC, (U > 4 ? 4 : U), 6>); break;
+      case 2: go(spmm_sparse_kernel<LPG, VEC, 2, 8>); break;
+      default: go(spmm_sparse_kernel<LPG, VEC, U, 4>); break;
+    }
     SR_CUDA_TRY(cudaGetLastError());
     if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;
@@ -613,23 +692,22 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
   constexpr int NCH_D = (LPG == 32) ? 1 : NCH;  // dense: whole K per pass unless K > 256
   if (P.n_units > 0) {
     const int TW = P.tile_cols;
-    const size_t smem = (size_t)kSddmmStages * StageLayout{TW * NCH_D * KC, P.trp_stride, true, kSddmmStages}.bytes() + kUnitColsBytes;
+    const size_t smem =
+        StageLayout{TW * NCH_D * KC, P.trp_stride, true, kSddmmStages, 0, true}.smem(kSddmmStages);
+    const unsigned grid = (unsigned)std::min<int64_t>(P.n_units, (int64_t)kDenseCtasPerSM * num_sms());
+    const int flags = (VEC == 4 ? 1 : 0) | (dense_dbg() << 1);
     auto launch = [&](auto kern) -> int {
       SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-      kern<<<(unsigned)P.n_units, (kDenseWarps + 1) * 32, smem, s>>>(
-          P.units.p, P.vtiles.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.d_oidx.p, P.pos_xrow.p, X, ldx, Y, ldy,
-          (int)K, TW, P.trp_stride, out);
+      kern<<<grid, (kDenseWarps + 1) * 32, smem, s>>>(
+          P.units.p, (int)P.n_units, P.vtiles.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.d_oidx.p, P.pos_xrow.p, X, ldx,
+          Y, ldy, (int)K, TW, P.trp_stride, out, flags);
       SR_CUDA_TRY(cudaGetLastError());
       return SR_OK;
     };
     constexpr int UD = 4;
     if (P.profiling) SR_TRY(prof_begin(P, 3, s));
-    if (VEC == 4) {
-      if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 8, true>));
-      else SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 16, true>));
-    } else {
-      SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 16, false>));
-    }
+    if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 8>));
+    else SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 16>));
     if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;
   }

@@ -141,6 +141,7 @@ struct DevPlan {
   int64_t dscratch_k = 0;
   DevBuf<int32_t> pos_xrow;   // position -> original row
   DevBuf<int32_t> pos_out;    // position -> SpMM output row
+  DevBuf<int32_t> dense_out;  // position -> SpMM output row if the row has dense nnz, else -1
   // phase S
   DevBuf<int2> s_ent;         // {col, __float_as_int(val)} remainder stream
   DevBuf<int32_t> s_oidx;     // SDDMM output index per remainder nnz

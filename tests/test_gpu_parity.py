@@ -274,22 +274,24 @@ def test_shard_simulation(env, oracle, world):
 
 # ------------------------------------------------------------------ full-size configs
 @pytest.mark.slow
-def test_rmat_full_size_sampled(env, oracle):
-    """C2 at its full size in the launch configuration bench.py times (K=128 and 32):
-    plan bit-exact vs the oracle, outputs checked on 2000 sampled rows / all SDDMM nnz of
-    those rows."""
+@pytest.mark.parametrize("config", ["rmat", "banded", "gnn", "cf"])
+def test_full_size_sampled(env, oracle, config):
+    """C2-C5 at full size in the launch configuration bench.py times (default plan
+    parameters, AUTO mode): plan bit-exact vs the oracle; SpMM checked on 2000 sampled rows
+    plus the 20 longest rows (K=128, and K=32 for C2); SDDMM on every nnz of those rows."""
     sr, torch = env
-    A = g.rmat()
+    A = g.make(config)
     kw = dict(siglen=128, bsize=2, seed=4, max_bucket=32, threshold_size=256, panel_rows=64, dense_min=2,
               mode=0)
     M = sr.SparseMatrix.from_csr(A)
     M.reorder(sr.default_params(**kw))
     ref = oracle.plan(A, **kw)
     _assert_plan_equal(M, ref)
+    del ref
     rng = np.random.default_rng(0)
     deg = np.diff(A.rowptr)
     rows = np.unique(np.concatenate([rng.integers(0, A.nrows, 2000), np.argsort(deg)[-20:]]))
-    for K in (128, 32):
+    for K in ((128, 32) if config == "rmat" else (128,)):
         B = g.dense(A.ncols, K)
         C = M.spmm(torch.from_numpy(B).cuda())
         torch.cuda.synchronize()
