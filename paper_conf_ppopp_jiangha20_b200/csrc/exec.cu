@@ -250,7 +250,7 @@ constexpr int kMaxStages = 3;   // SpMM runs 3 stages, SDDMM 2 (its stages also 
 constexpr int kSpmmStages = 3;
 constexpr int kSddmmStages = 2;
 constexpr int kDenseCtasPerSM = 2;
-constexpr size_t kUnitColsBytes = (size_t)kMaxUnitTiles * kMaxExecTile * 4;
+constexpr size_t kUnitBlobBytes = kMaxUnitBlobBytes;  // DUnit + VTiles + dense column ids
 
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
@@ -279,7 +279,7 @@ struct StageLayout {
   __host__ __device__ size_t ent_off() const { return trp_off() + (size_t)trp_ints * 4; }
   __host__ __device__ size_t oidx_off() const { return ent_off() + (size_t)kMaxTileEntries * 8; }
   __host__ __device__ size_t bytes() const { return oidx_off() + (oidx ? (size_t)kMaxTileEntries * 4 : 0); }
-  __host__ size_t smem(int nst_) const { return (size_t)nst_ * bytes() + kUnitColsBytes; }
+  __host__ size_t smem(int nst_) const { return (size_t)nst_ * bytes() + 2 * kUnitBlobBytes; }
 };
 
 // Producer warp: every tile of every unit of this CTA.
@@ -289,23 +289,36 @@ __device__ __forceinline__ void dense_produce(const DUnit* __restrict__ units, i
                                               const int32_t* __restrict__ trp, const int2* __restrict__ ent,
                                               const int32_t* __restrict__ oidx, const float* __restrict__ src,
                                               int64_t ld, int K, int KCP, const StageLayout& L, char* smem,
-                                              uint64_t* full, uint64_t* empty) {
+                                              uint64_t* full, uint64_t* empty, const int4* __restrict__ blobs,
+                                              const int2* __restrict__ blob_meta, uint64_t* blob_bar) {
   const int lane = threadIdx.x & 31;
   const size_t SB = L.bytes();
-  int32_t* ucols = reinterpret_cast<int32_t*>(smem + L.nst * SB);
   const int npass = (K + KCP - 1) / KCP;
+  // This CTA's units are blockIdx.x + k·gridDim.x (units are sorted by decreasing size, so the
+  // round robin balances).  Everything the producer needs about a unit — its DUnit, its
+  // VTiles and its dense column ids — is one contiguous 16-byte-aligned blob, fetched by one
+  // bulk copy two units ahead into a 2-slot ring: no dependent global load on the issue path.
+  char* ring = smem + L.nst * SB;
+  const int nmine = ((int)blockIdx.x < n_units) ? (n_units - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x : 0;
+  auto fetch_blob = [&](int k, int2 m) {
+    if (lane == 0) {
+      mbar_expect_tx(&blob_bar[k & 1], (uint32_t)m.y);
+      bulk_g2s(ring + (k & 1) * kUnitBlobBytes, reinterpret_cast<const char*>(blobs) + (int64_t)m.x * 16,
+               (uint32_t)m.y, &blob_bar[k & 1]);
+    }
+  };
+  for (int k = 0; k < 2 && k < nmine; ++k) fetch_blob(k, blob_meta[blockIdx.x + k * gridDim.x]);
+  int2 m_next = (2 < nmine) ? blob_meta[blockIdx.x + 2 * gridDim.x] : make_int2(0, 0);
   int idx = 0;
-  for (int uid = blockIdx.x; uid < n_units; uid += gridDim.x) {
-    const DUnit u = units[uid];
-    const bool last_unit = uid + (int)gridDim.x >= n_units;
-    // the unit's tile descriptors (lane i holds tile i) and its dense column ids (contiguous,
-    // <= kMaxUnitTiles·kMaxExecTile) are fetched once per unit
-    const VTile mine = lane < u.nvt ? vtiles[u.vt0 + lane] : VTile{0, 0, 0, 0};
+  for (int k = 0; k < nmine; ++k) {
+    const int uid = blockIdx.x + k * gridDim.x;
+    mbar_wait(&blob_bar[k & 1], (k >> 1) & 1);
+    const char* blob = ring + (k & 1) * kUnitBlobBytes;
+    const DUnit u = *reinterpret_cast<const DUnit*>(blob);
+    const bool last_unit = k == nmine - 1;
+    const VTile mine = lane < u.nvt ? reinterpret_cast<const VTile*>(blob + sizeof(DUnit))[lane] : VTile{0, 0, 0, 0};
     const int col_lo = __shfl_sync(FULL, mine.col0, 0);
-    const int last_col0 = __shfl_sync(FULL, mine.col0, u.nvt - 1), last_nc = __shfl_sync(FULL, mine.ncols, u.nvt - 1);
-    const int ncol_unit = last_col0 + last_nc - col_lo;
-    for (int j = lane; j < ncol_unit; j += 32) ucols[j] = dense_cols[col_lo + j];
-    __syncwarp();
+    const int32_t* ucols = reinterpret_cast<const int32_t*>(blob + sizeof(DUnit) + u.nvt * sizeof(VTile));
     for (int pass = 0; pass < npass; ++pass) {
       const int k0 = pass * KCP, kw = min(KCP, K - k0);
       for (int ti = 0; ti < u.nvt; ++ti, ++idx) {
@@ -365,8 +378,15 @@ __device__ __forceinline__ void dense_produce(const DUnit* __restrict__ units, i
           bulk_g2s(base + L.oidx_off(), oidx + v.ent0, (uint32_t)(v.nent * 4), &full[st]);
       }
     }
-    __syncwarp();
+    __syncwarp();  // every lane is done with this blob slot
+    if (k + 2 < nmine) {
+      fetch_blob(k + 2, m_next);
+      m_next = (k + 3 < nmine) ? blob_meta[blockIdx.x + (k + 3) * gridDim.x] : make_int2(0, 0);
+    }
   }
+  (void)units;
+  (void)vtiles;
+  (void)dense_cols;
 }
 
 __device__ __forceinline__ void dense_init_barriers(uint64_t* full, uint64_t* empty) {
@@ -375,6 +395,8 @@ __device__ __forceinline__ void dense_init_barriers(uint64_t* full, uint64_t* em
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], kDenseWarps);
     }
+    mbar_init(&full[kMaxStages], 1);  // unit-blob ring (producer only)
+    mbar_init(&full[kMaxStages + 1], 1);
     fence_mbar_init();
   }
   __syncthreads();
@@ -387,18 +409,19 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) spmm_
     const int32_t* __restrict__ dense_cols, const int32_t* __restrict__ trp, const int2* __restrict__ ent,
     const int32_t* __restrict__ dense_out, const float* __restrict__ B, int64_t ldb, float* __restrict__ C,
     int64_t ldc, int K, int TW, int TS, int P, float* __restrict__ scratch, const int2* __restrict__ split_info,
-    int* __restrict__ split_counter, int dbg) {
+    int* __restrict__ split_counter, const int4* __restrict__ blobs, const int2* __restrict__ blob_meta, int dbg) {
   constexpr int G = 32 / LPG;
   constexpr int KC = LPG * VEC;
   extern __shared__ __align__(128) char smem[];
-  __shared__ uint64_t full[kMaxStages], empty[kMaxStages];
+  __shared__ uint64_t full[kMaxStages + 2], empty[kMaxStages];
   __shared__ int last_ticket;
   const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
   const int warp = threadIdx.x >> 5;
   const StageLayout L{TW * KC, TS, false, kSpmmStages, dbg >> 1, (dbg & 1) != 0};
   dense_init_barriers(full, empty);
   if (warp == kDenseWarps) {
-    dense_produce(units, n_units, vtiles, dense_cols, trp, ent, nullptr, B, ldb, K, KC, L, smem, full, empty);
+    dense_produce(units, n_units, vtiles, dense_cols, trp, ent, nullptr, B, ldb, K, KC, L, smem, full, empty,
+                  blobs, blob_meta, full + kMaxStages);
     return;
   }
   const size_t SB = L.bytes();
@@ -504,18 +527,19 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) sddmm
     const int32_t* __restrict__ dense_cols, const int32_t* __restrict__ trp, const int2* __restrict__ ent,
     const int32_t* __restrict__ d_oidx, const int32_t* __restrict__ pos_xrow, const float* __restrict__ X,
     int64_t ldx, const float* __restrict__ Y, int64_t ldy, int K, int TW, int TS, float* __restrict__ out,
-    int dbg) {
+    const int4* __restrict__ blobs, const int2* __restrict__ blob_meta, int dbg) {
   constexpr int G = 32 / LPG;
   constexpr int KC = LPG * VEC;   // columns of one chunk
   constexpr int KCP = NCH * KC;   // columns staged per pass (slot stride)
   extern __shared__ __align__(128) char smem[];
-  __shared__ uint64_t full[kMaxStages], empty[kMaxStages];
+  __shared__ uint64_t full[kMaxStages + 2], empty[kMaxStages];
   const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
   const int warp = threadIdx.x >> 5;
   const StageLayout L{TW * KCP, TS, true, kSddmmStages, dbg >> 1, (dbg & 1) != 0};
   dense_init_barriers(full, empty);
   if (warp == kDenseWarps) {
-    dense_produce(units, n_units, vtiles, dense_cols, trp, ent, d_oidx, Y, ldy, K, KCP, L, smem, full, empty);
+    dense_produce(units, n_units, vtiles, dense_cols, trp, ent, d_oidx, Y, ldy, K, KCP, L, smem, full, empty,
+                  blobs, blob_meta, full + kMaxStages);
     return;
   }
   const size_t SB = L.bytes();
@@ -649,7 +673,8 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
       SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
       kern<<<grid, (kDenseWarps + 1) * 32, smem, s>>>(
           P.units.p, (int)P.n_units, P.vtiles.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.dense_out.p, B, ldb, C, ldc,
-          (int)K, TW, P.trp_stride, P.panel_rows, P.dscratch.p, P.dsplit_info.p, P.dsplit_counter.p, flags);
+          (int)K, TW, P.trp_stride, P.panel_rows, P.dscratch.p, P.dsplit_info.p, P.dsplit_counter.p, P.blobs.p,
+          P.blob_meta.p, flags);
       SR_CUDA_TRY(cudaGetLastError());
       return SR_OK;
     };
@@ -670,11 +695,13 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
       kern<<<grid, kSparseWarps * 32, 0, s>>>(P.items.p, P.item_meta.p, P.n_items, P.s_ent.p, B, ldb, C, ldc, (int)K,
                                                P.scratch.p, P.split_info.p, P.split_counter.p);
     };
-    // SR_SPARSE_VARIANT (tuning knob): 0 = U 8 / 4 CTAs per SM (default), 1 = U 4 / 6, 2 = U 2 / 8
+    // occupancy beats per-warp memory parallelism here (profiles/r01): U=2 gathers per lane
+    // at 8 CTAs (64 warps) per SM.  SR_SPARSE_VARIANT (tuning knob): 1 = U 4 / 6 CTAs,
+    // 3 = U 8 / 4 CTAs.
     switch (sparse_variant()) {
       case 1: go(spmm_sparse_kernel<LPG, VEC, (U > 4 ? 4 : U), 6>); break;
-      case 2: go(spmm_sparse_kernel<LPG, VEC, 2, 8>); break;
-      default: go(spmm_sparse_kernel<LPG, VEC, U, 4>); break;
+      case 3: go(spmm_sparse_kernel<LPG, VEC, U, 4>); break;
+      default: go(spmm_sparse_kernel<LPG, VEC, 2, 8>); break;
     }
     SR_CUDA_TRY(cudaGetLastError());
     if (P.profiling) SR_TRY(prof_end(P, s));
@@ -700,7 +727,7 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
       SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
       kern<<<grid, (kDenseWarps + 1) * 32, smem, s>>>(
           P.units.p, (int)P.n_units, P.vtiles.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.d_oidx.p, P.pos_xrow.p, X, ldx,
-          Y, ldy, (int)K, TW, P.trp_stride, out, flags);
+          Y, ldy, (int)K, TW, P.trp_stride, out, P.blobs.p, P.blob_meta.p, flags);
       SR_CUDA_TRY(cudaGetLastError());
       return SR_OK;
     };

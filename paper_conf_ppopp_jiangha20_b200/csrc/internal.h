@@ -121,6 +121,8 @@ struct __align__(16) DUnit {
 constexpr int kMaxUnitTiles = 16;
 constexpr int kMaxExecTile = 64;
 constexpr int kMaxTileEntries = 512;
+// producer-side record of a unit: DUnit, its VTiles, its dense column ids (16-byte aligned)
+constexpr int kMaxUnitBlobBytes = 32 + kMaxUnitTiles * 16 + kMaxUnitTiles * kMaxExecTile * 4;
 
 // Device-resident execution plan.
 struct DevPlan {
@@ -129,6 +131,8 @@ struct DevPlan {
   int64_t n_units = 0;
   DevBuf<int32_t> dense_cols;
   DevBuf<VTile> vtiles;
+  DevBuf<int4> blobs;         // per unit: DUnit | VTile[nvt] | dense column ids (16-byte records)
+  DevBuf<int2> blob_meta;     // per unit: {offset in 16-byte words, bytes}
   DevBuf<int32_t> trp;        // per virtual tile: trp_stride offsets relative to its entry block
   int32_t trp_stride = 68;
   DevBuf<int32_t> drow_ptr;   // positions -> dense nnz offsets (only "row has dense nnz" is used)
