@@ -91,6 +91,9 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
       : "memory");
 }
 
+// (An L2 evict_last / evict_first split of the gathered rows by access count was measured in
+// round 1 and did not help: profiles/r01/NOTES.md.)
+
 // ------------------------------------------------------------------ phase S: SpMM
 template <int LPG, int VEC, int U, int MINB = 4>
 __global__ void __launch_bounds__(256, MINB) spmm_sparse_kernel(
@@ -120,11 +123,11 @@ __global__ void __launch_bounds__(256, MINB) spmm_sparse_kernel(
         for (int u = 0; u < U; ++u) {
           const int j = base + u * G + g;
           const int src = j & 31;
-          const int c = __shfl_sync(FULL, my.x, src);
+          const int cf = __shfl_sync(FULL, my.x, src);
           const float v = __int_as_float(__shfl_sync(FULL, my.y, src));
           const bool ok = (j < n) && kv;
           a[u] = ok ? v : 0.f;
-          if (ok) b[u].load_g(B + (int64_t)c * ldb + kk); else b[u].zero();
+          if (ok) b[u].load_g(B + (int64_t)cf * ldb + kk); else b[u].zero();
         }
 #pragma unroll
         for (int u = 0; u < U; ++u) acc.fma(a[u], b[u]);
@@ -179,8 +182,8 @@ __global__ void __launch_bounds__(256, MINB) spmm_sparse_kernel(
 }
 
 // ------------------------------------------------------------------ phase S: SDDMM
-template <int LPG, int VEC, int U, int NCH>
-__global__ void __launch_bounds__(256) sddmm_sparse_kernel(
+template <int LPG, int VEC, int U, int NCH, int MINB = 4>
+__global__ void __launch_bounds__(256, MINB) sddmm_sparse_kernel(
     const Item* __restrict__ items, int64_t n_items, const int2* __restrict__ ent,
     const int32_t* __restrict__ oidx, const float* __restrict__ X, int64_t ldx,
     const float* __restrict__ Y, int64_t ldy, int K, float* __restrict__ out) {
@@ -517,6 +520,103 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) spmm_
   }
 }
 
+// SpMM dense tiles through L1 instead of shared memory ("L1 staging"): one CTA per unit, its
+// warps walk the unit's tiles without any barrier and gather the dense columns' B rows with
+// L1-allocating 128-bit loads; the first warp to touch a dense column brings its row into
+// L1 and the other rows of the panel hit it there (the reuse ASpT gets from shared memory).
+// Entries carry their global column id (d_col, tile-major like d_ent).
+template <int LPG, int VEC, int U, int RPW>
+__global__ void __launch_bounds__(kDenseWarps * 32, 4) spmm_dense_l1_kernel(
+    const DUnit* __restrict__ units, const VTile* __restrict__ vtiles, const int32_t* __restrict__ trp,
+    const int2* __restrict__ ent, const int32_t* __restrict__ dcol, const int32_t* __restrict__ dense_out,
+    const float* __restrict__ B, int64_t ldb, float* __restrict__ C, int64_t ldc, int K, int TS, int P,
+    float* __restrict__ scratch, const int2* __restrict__ split_info, int* __restrict__ split_counter) {
+  constexpr int G = 32 / LPG;
+  constexpr int KC = LPG * VEC;
+  __shared__ int last_ticket;
+  const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
+  const int warp = threadIdx.x >> 5;
+  const DUnit u = units[blockIdx.x];
+  const int r0 = warp * RPW;
+  const int out_row = (lane < RPW && r0 + lane < u.nrows) ? dense_out[u.q0 + r0 + lane] : -1;
+  for (int k0 = 0; k0 < K; k0 += KC) {
+    const int kk = k0 + lg * VEC;
+    const bool kv = kk < K;
+    Frag<VEC> acc[RPW];
+#pragma unroll
+    for (int i = 0; i < RPW; ++i) acc[i].zero();
+    if (r0 < u.nrows) {
+      for (int t = 0; t < u.nvt; ++t) {
+        const int vt = u.vt0 + t;
+        const int ent0 = __ldg(&vtiles[vt].ent0);
+        const int bnd = lane <= RPW ? __ldg(trp + (int64_t)vt * TS + r0 + lane) : 0;
+        const int e_lo = __shfl_sync(FULL, bnd, 0), e_hi = __shfl_sync(FULL, bnd, RPW);
+        for (int e = e_lo; e < e_hi; e += 32) {
+          const int n = min(32, e_hi - e);
+          const int2 my = lane < n ? __ldcs(ent + ent0 + e + lane) : make_int2(0, 0);
+          const int myc = lane < n ? __ldcs(dcol + ent0 + e + lane) : 0;
+#pragma unroll
+          for (int i = 0; i < RPW; ++i) {
+            const int a = max(0, __shfl_sync(FULL, bnd, i) - e), b = min(n, __shfl_sync(FULL, bnd, i + 1) - e);
+            for (int base = a; base < b; base += G * U) {
+              Frag<VEC> bv[U];
+              float av[U];
+#pragma unroll
+              for (int uu = 0; uu < U; ++uu) {
+                const int j = base + uu * G + g;
+                const int c = __shfl_sync(FULL, myc, j & 31);
+                const float v = __int_as_float(__shfl_sync(FULL, my.y, j & 31));
+                const bool ok = j < b && kv;
+                av[uu] = ok ? v : 0.f;
+                if (ok) bv[uu].load_g(B + (int64_t)c * ldb + kk); else bv[uu].zero();
+              }
+#pragma unroll
+              for (int uu = 0; uu < U; ++uu) acc[i].fma(av[uu], bv[uu]);
+            }
+          }
+        }
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < RPW; ++i) {
+#pragma unroll
+      for (int off = LPG; off < 32; off <<= 1) acc[i].xor_add(off);
+      const int orow = __shfl_sync(FULL, out_row, i);
+      if (r0 + i < u.nrows && g == 0 && kv) {
+        if (u.split >= 0)
+          acc[i].store(scratch + ((int64_t)u.split * P + r0 + i) * K + kk);
+        else if (orow >= 0)
+          acc[i].store_cs(C + (int64_t)orow * ldc + kk);
+      }
+    }
+  }
+  if (u.split >= 0) {
+    __threadfence();
+    __syncthreads();
+    const int2 si = split_info[u.split];
+    if (threadIdx.x == 0) last_ticket = (atomicAdd(split_counter + si.x, 1) == si.y - 1);
+    __syncthreads();
+    if (!last_ticket) return;
+    __threadfence();
+    for (int i = 0; i < RPW; ++i) {
+      const int orow = __shfl_sync(FULL, out_row, i);
+      if (r0 + i >= u.nrows || orow < 0) continue;
+      for (int k = lane * VEC; k < K; k += 32 * VEC) {
+        Frag<VEC> s;
+        s.zero();
+        for (int c = 0; c < si.y; ++c) {
+          Frag<VEC> part;
+          part.load_cg(scratch + ((int64_t)(si.x + c) * P + r0 + i) * K + k);
+          s.add(part);
+        }
+        s.store_cs(C + (int64_t)orow * ldc + k);
+      }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) split_counter[si.x] = 0;
+  }
+}
+
 // SDDMM dense tiles.  Lane geometry as phase S: LPG lanes × NCH chunks of LPG·VEC columns
 // cover one nnz (K=128: 8 lanes × 4 float4, 4 nnz per warp step, 3-step shuffle reduction).
 // X fragments of the current row come from global memory (L1-resident across the tiles);
@@ -634,6 +734,14 @@ int dense_dbg() {
   return v;
 }
 
+int dense_engine() {
+  static const int v = [] {
+    const char* d = getenv("SR_DENSE_ENGINE");
+    return (d && std::string(d) == "l1") ? 1 : 0;
+  }();
+  return v;
+}
+
 int sparse_variant() {
   static const int v = [] {
     const char* d = getenv("SR_SPARSE_VARIANT");
@@ -679,8 +787,21 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
       return SR_OK;
     };
     if (P.profiling) SR_TRY(prof_begin(P, 1, s));
-    if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 8>));
-    else SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 16>));
+    if (dense_engine() == 1) {  // L1 staging (SR_DENSE_ENGINE=l1)
+      auto l1 = [&](auto kern) -> int {
+        kern<<<(unsigned)P.n_units, kDenseWarps * 32, 0, s>>>(
+            P.units.p, P.vtiles.p, P.trp.p, P.d_ent.p, P.d_col.p, P.dense_out.p, B, ldb, C, ldc, (int)K,
+            P.trp_stride, P.panel_rows, P.dscratch.p, P.dsplit_info.p, P.dsplit_counter.p);
+        SR_CUDA_TRY(cudaGetLastError());
+        return SR_OK;
+      };
+      if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(l1(spmm_dense_l1_kernel<LPG, VEC, 2, 8>));
+      else SR_TRY(l1(spmm_dense_l1_kernel<LPG, VEC, 2, 16>));
+    } else if (P.panel_rows <= 8 * kDenseWarps) {
+      SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 8>));
+    } else {
+      SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 16>));
+    }
     if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;
   }
@@ -741,8 +862,16 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
   if (P.n_sitems > 0) {
     const unsigned grid = (unsigned)((P.n_sitems + kSparseWarps - 1) / kSparseWarps);
     if (P.profiling) SR_TRY(prof_begin(P, 4, s));
-    sddmm_sparse_kernel<LPG, VEC, U, NCH><<<grid, kSparseWarps * 32, 0, s>>>(
-        P.items.p, P.n_sitems, P.s_ent.p, P.s_oidx.p, X, ldx, Y, ldy, (int)K, out);
+    auto go = [&](auto kern) {
+      kern<<<grid, kSparseWarps * 32, 0, s>>>(P.items.p, P.n_sitems, P.s_ent.p, P.s_oidx.p, X, ldx, Y, ldy, (int)K,
+                                               out);
+    };
+    // SR_SPARSE_VARIANT (tuning knob) also selects the SDDMM occupancy point
+    switch (sparse_variant()) {
+      case 1: go(sddmm_sparse_kernel<LPG, VEC, U, NCH, 1>); break;
+      case 2: go(sddmm_sparse_kernel<LPG, VEC, 1, NCH, 6>); break;
+      default: go(sddmm_sparse_kernel<LPG, VEC, U, NCH, 4>); break;
+    }
     SR_CUDA_TRY(cudaGetLastError());
     if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;

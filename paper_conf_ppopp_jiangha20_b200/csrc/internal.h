@@ -118,9 +118,9 @@ struct __align__(16) DUnit {
   int32_t split;      // -1: the unit covers its whole panel; else its partial-sum slot
   int32_t pad0, pad1, pad2;
 };
-constexpr int kMaxUnitTiles = 16;
+constexpr int kMaxUnitTiles = 8;
 constexpr int kMaxExecTile = 64;
-constexpr int kMaxTileEntries = 512;
+constexpr int kMaxTileEntries = 384;  // SpMM: 3 stages + blob ring must fit twice per SM
 // producer-side record of a unit: DUnit, its VTiles, its dense column ids (16-byte aligned)
 constexpr int kMaxUnitBlobBytes = 32 + kMaxUnitTiles * 16 + kMaxUnitTiles * kMaxExecTile * 4;
 
@@ -138,6 +138,7 @@ struct DevPlan {
   DevBuf<int32_t> drow_ptr;   // positions -> dense nnz offsets (only "row has dense nnz" is used)
   DevBuf<int2> d_ent;         // tile-major {slot in tile, __float_as_int(val)}
   DevBuf<int32_t> d_oidx;     // SDDMM output index per dense nnz (tile-major)
+  DevBuf<int32_t> d_col;      // global column id per dense nnz (tile-major; L1-staging kernel)
   DevBuf<int2> dsplit_info;   // per split unit: {first slot, nchunks}
   DevBuf<int32_t> dsplit_counter;
   int64_t n_dslots = 0;
