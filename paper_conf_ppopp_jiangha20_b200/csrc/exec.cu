@@ -12,6 +12,9 @@
 //   are in flight per lane.  SDDMM reduces each dot product with warp shuffles.
 // Lane geometry: LPG lanes cover LPG·VEC columns of one nnz; G = 32/LPG groups of a warp
 //   work on G different nnz at once (K = 32 -> 4 nnz per warp instruction).
+#include <cuda.h>  // CUtensorMap
+#include <cudaTypedefs.h>  // PFN_cuTensorMapEncodeTiled
+
 #include <algorithm>
 
 #include "internal.h"
@@ -93,6 +96,21 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 
 // (An L2 evict_last / evict_first split of the gathered rows by access count was measured in
 // round 1 and did not help: profiles/r01/NOTES.md.)
+
+// TMA tile::gather4 (sm_100): rows r0..r3 of a 2-D tensor map, box = {columns, 1}, into 4
+// consecutive box-sized rows of shared memory (128-byte aligned destination).
+__device__ __forceinline__ void tma_gather4(void* dst, const CUtensorMap* map, int col, int r0, int r1, int r2,
+                                            int r3, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(col), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(smem_u32(bar))
+      : "memory");
+}
+
+__device__ __forceinline__ char* align128(char* p) {
+  return p + ((128 - (smem_u32(p) & 127)) & 127);
+}
 
 // ------------------------------------------------------------------ phase S: SpMM
 template <int LPG, int VEC, int U, int MINB = 4>
@@ -277,12 +295,14 @@ struct StageLayout {
   int nst;        // pipeline depth (<= kMaxStages)
   int dbg;        // measurement knobs (SR_DEBUG_DENSE): 1 = skip consumer math, 2 = skip copies
   bool bulk;      // TMA bulk copies (16-byte-aligned rows); else the producer copies with LDG/STS
-  __host__ __device__ size_t b_off() const { return sizeof(StageHdr); }
+  // stage = [staged rows (128-byte aligned for the tensor TMA)] [trp] [entries] [oidx] [header]
+  __host__ __device__ size_t b_off() const { return 0; }
   __host__ __device__ size_t trp_off() const { return b_off() + (size_t)b_floats * 4; }
   __host__ __device__ size_t ent_off() const { return trp_off() + (size_t)trp_ints * 4; }
   __host__ __device__ size_t oidx_off() const { return ent_off() + (size_t)kMaxTileEntries * 8; }
-  __host__ __device__ size_t bytes() const { return oidx_off() + (oidx ? (size_t)kMaxTileEntries * 4 : 0); }
-  __host__ size_t smem(int nst_) const { return (size_t)nst_ * bytes() + 2 * kUnitBlobBytes; }
+  __host__ __device__ size_t hdr_off() const { return oidx_off() + (oidx ? (size_t)kMaxTileEntries * 4 : 0); }
+  __host__ __device__ size_t bytes() const { return (hdr_off() + sizeof(StageHdr) + 127) / 128 * 128; }
+  __host__ size_t smem(int nst_) const { return 128 + (size_t)nst_ * bytes() + 2 * kUnitBlobBytes; }
 };
 
 // Producer warp: every tile of every unit of this CTA.
@@ -293,7 +313,8 @@ __device__ __forceinline__ void dense_produce(const DUnit* __restrict__ units, i
                                               const int32_t* __restrict__ oidx, const float* __restrict__ src,
                                               int64_t ld, int K, int KCP, const StageLayout& L, char* smem,
                                               uint64_t* full, uint64_t* empty, const int4* __restrict__ blobs,
-                                              const int2* __restrict__ blob_meta, uint64_t* blob_bar) {
+                                              const int2* __restrict__ blob_meta, uint64_t* blob_bar,
+                                              const CUtensorMap* tmap) {
   const int lane = threadIdx.x & 31;
   const size_t SB = L.bytes();
   const int npass = (K + KCP - 1) / KCP;
@@ -334,7 +355,7 @@ __device__ __forceinline__ void dense_produce(const DUnit* __restrict__ units, i
         v.ncols = __shfl_sync(FULL, mine.ncols, ti);
         char* base = smem + st * SB;
         if (lane == 0) {
-          StageHdr* h = reinterpret_cast<StageHdr*>(base);
+          StageHdr* h = reinterpret_cast<StageHdr*>(base + L.hdr_off());
           int f = 0;
           if (ti == 0) f |= kFirstOfPass;
           if (ti == u.nvt - 1) f |= kLastOfPass;
@@ -366,14 +387,27 @@ __device__ __forceinline__ void dense_produce(const DUnit* __restrict__ units, i
           if (lane == 0) mbar_arrive(&full[st]);
           continue;
         }
-        const uint32_t bytes =
-            (uint32_t)(v.ncols * kw * 4 + L.trp_ints * 4 + v.nent * 8 + (L.oidx ? v.nent * 4 : 0));
+        const uint32_t row_bytes = tmap ? (uint32_t)(((v.ncols + 3) & ~3) * KCP * 4) : (uint32_t)(v.ncols * kw * 4);
+        const uint32_t bytes = row_bytes + (uint32_t)(L.trp_ints * 4 + v.nent * 8 + (L.oidx ? v.nent * 4 : 0));
         if (lane == 0) mbar_expect_tx(&full[st], bytes);
         __syncwarp();
         const int32_t* cols = ucols + (v.col0 - col_lo);
-        for (int j = lane; j < v.ncols; j += 32)
-          bulk_g2s(base + L.b_off() + (size_t)j * KCP * 4, src + (int64_t)cols[j] * ld + k0, (uint32_t)(kw * 4),
-                   &full[st]);
+        if (tmap) {
+          // TMA gather4: one instruction stages four dense-column rows (box = KCP columns × 1 row
+          // of the row-major operand, 4 row coordinates); a ragged last group repeats a row
+          for (int j4 = lane; j4 * 4 < v.ncols; j4 += 32) {
+            const int j = j4 * 4;
+            const int c0 = cols[j];
+            const int c1 = j + 1 < v.ncols ? cols[j + 1] : c0;
+            const int c2 = j + 2 < v.ncols ? cols[j + 2] : c0;
+            const int c3 = j + 3 < v.ncols ? cols[j + 3] : c0;
+            tma_gather4(base + L.b_off() + (size_t)j * KCP * 4, tmap, k0, c0, c1, c2, c3, &full[st]);
+          }
+        } else {
+          for (int j = lane; j < v.ncols; j += 32)
+            bulk_g2s(base + L.b_off() + (size_t)j * KCP * 4, src + (int64_t)cols[j] * ld + k0, (uint32_t)(kw * 4),
+                     &full[st]);
+        }
         if (lane == 0)
           bulk_g2s(base + L.trp_off(), trp + (int64_t)vt * L.trp_ints, (uint32_t)(L.trp_ints * 4), &full[st]);
         if (lane == 1 && v.nent > 0) bulk_g2s(base + L.ent_off(), ent + v.ent0, (uint32_t)(v.nent * 8), &full[st]);
@@ -412,19 +446,21 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) spmm_
     const int32_t* __restrict__ dense_cols, const int32_t* __restrict__ trp, const int2* __restrict__ ent,
     const int32_t* __restrict__ dense_out, const float* __restrict__ B, int64_t ldb, float* __restrict__ C,
     int64_t ldc, int K, int TW, int TS, int P, float* __restrict__ scratch, const int2* __restrict__ split_info,
-    int* __restrict__ split_counter, const int4* __restrict__ blobs, const int2* __restrict__ blob_meta, int dbg) {
+    int* __restrict__ split_counter, const int4* __restrict__ blobs, const int2* __restrict__ blob_meta,
+    const __grid_constant__ CUtensorMap tmap, int use_tmap, int dbg) {
   constexpr int G = 32 / LPG;
   constexpr int KC = LPG * VEC;
-  extern __shared__ __align__(128) char smem[];
+  extern __shared__ __align__(128) char smem_raw[];
+  char* const smem = align128(smem_raw);
   __shared__ uint64_t full[kMaxStages + 2], empty[kMaxStages];
   __shared__ int last_ticket;
   const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
   const int warp = threadIdx.x >> 5;
-  const StageLayout L{TW * KC, TS, false, kSpmmStages, dbg >> 1, (dbg & 1) != 0};
+  const StageLayout L{((TW + 3) & ~3) * KC, TS, false, kSpmmStages, dbg >> 1, (dbg & 1) != 0};
   dense_init_barriers(full, empty);
   if (warp == kDenseWarps) {
     dense_produce(units, n_units, vtiles, dense_cols, trp, ent, nullptr, B, ldb, K, KC, L, smem, full, empty,
-                  blobs, blob_meta, full + kMaxStages);
+                  blobs, blob_meta, full + kMaxStages, use_tmap ? &tmap : nullptr);
     return;
   }
   const size_t SB = L.bytes();
@@ -435,7 +471,7 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) spmm_
     const int st = idx % L.nst;
     mbar_wait(&full[st], (idx / L.nst) & 1);
     const char* base = smem + st * SB;
-    const StageHdr hd = *reinterpret_cast<const StageHdr*>(base);
+    const StageHdr hd = *reinterpret_cast<const StageHdr*>(base + L.hdr_off());
     if (hd.flags & kFirstOfUnit)
       out_row = (lane < RPW && r0 + lane < hd.nrows) ? dense_out[hd.q0 + r0 + lane] : -1;
     if (hd.flags & kFirstOfPass) {
@@ -627,19 +663,21 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) sddmm
     const int32_t* __restrict__ dense_cols, const int32_t* __restrict__ trp, const int2* __restrict__ ent,
     const int32_t* __restrict__ d_oidx, const int32_t* __restrict__ pos_xrow, const float* __restrict__ X,
     int64_t ldx, const float* __restrict__ Y, int64_t ldy, int K, int TW, int TS, float* __restrict__ out,
-    const int4* __restrict__ blobs, const int2* __restrict__ blob_meta, int dbg) {
+    const int4* __restrict__ blobs, const int2* __restrict__ blob_meta, const __grid_constant__ CUtensorMap tmap,
+    int use_tmap, int dbg) {
   constexpr int G = 32 / LPG;
   constexpr int KC = LPG * VEC;   // columns of one chunk
   constexpr int KCP = NCH * KC;   // columns staged per pass (slot stride)
-  extern __shared__ __align__(128) char smem[];
+  extern __shared__ __align__(128) char smem_raw[];
+  char* const smem = align128(smem_raw);
   __shared__ uint64_t full[kMaxStages + 2], empty[kMaxStages];
   const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
   const int warp = threadIdx.x >> 5;
-  const StageLayout L{TW * KCP, TS, true, kSddmmStages, dbg >> 1, (dbg & 1) != 0};
+  const StageLayout L{((TW + 3) & ~3) * KCP, TS, true, kSddmmStages, dbg >> 1, (dbg & 1) != 0};
   dense_init_barriers(full, empty);
   if (warp == kDenseWarps) {
     dense_produce(units, n_units, vtiles, dense_cols, trp, ent, d_oidx, Y, ldy, K, KCP, L, smem, full, empty,
-                  blobs, blob_meta, full + kMaxStages);
+                  blobs, blob_meta, full + kMaxStages, use_tmap ? &tmap : nullptr);
     return;
   }
   const size_t SB = L.bytes();
@@ -649,7 +687,7 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) sddmm
     const int st = idx % L.nst;
     mbar_wait(&full[st], (idx / L.nst) & 1);
     const char* base = smem + st * SB;
-    const StageHdr hd = *reinterpret_cast<const StageHdr*>(base);
+    const StageHdr hd = *reinterpret_cast<const StageHdr*>(base + L.hdr_off());
     if (hd.flags & kFirstOfUnit) xrow = (lane < RPW && r0 + lane < hd.nrows) ? pos_xrow[hd.q0 + r0 + lane] : 0;
     if (!(L.dbg & 1) && r0 < hd.nrows) {
       const float* tile = reinterpret_cast<const float*>(base + L.b_off());
@@ -734,6 +772,37 @@ int dense_dbg() {
   return v;
 }
 
+// Tensor map of a row-major fp32 operand [rows × K] (leading dimension ld) for tile::gather4:
+// box = `box_cols` columns × 1 row.  The driver's encoder is reached through the runtime's
+// entry-point query, so libsr does not link libcuda.  SR_GATHER4=0 falls back to per-row
+// cp.async.bulk copies.  Returns false when TMA cannot describe the operand.
+bool make_row_gather_map(CUtensorMap* map, const float* base, int64_t rows, int64_t K, int64_t ld, int box_cols) {
+  static PFN_cuTensorMapEncodeTiled_v12000 encode = [] {
+    const char* e = getenv("SR_GATHER4");
+    if (e && std::string(e) == "0") return (PFN_cuTensorMapEncodeTiled_v12000) nullptr;
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess) {
+      cudaGetLastError();
+      return (PFN_cuTensorMapEncodeTiled_v12000) nullptr;
+    }
+    return reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  }();
+  // gather4 writes 4 box rows per instruction to a 128-byte-aligned destination: the staged
+  // row stride (box_cols floats) must keep 4-row groups 128-byte aligned
+  if (!encode || rows < 1 || rows >= (1ll << 31) || box_cols > 256 || (box_cols * 16) % 128 != 0 ||
+      ((uintptr_t)base % 16) != 0 || (ld * 4) % 16 != 0)
+    return false;
+  cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)(ld * 4)};
+  cuuint32_t box[2] = {(cuuint32_t)box_cols, 1};
+  cuuint32_t estr[2] = {1, 1};
+  return encode(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box, estr,
+                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 int dense_engine() {
   static const int v = [] {
     const char* d = getenv("SR_DENSE_ENGINE");
@@ -770,7 +839,10 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
   constexpr int UD = 4;                   // shared-memory reads in flight per lane (phase D)
   if (P.n_units > 0) {
     const int TW = P.tile_cols;
-    const size_t smem = StageLayout{TW * KC, P.trp_stride, false, kSpmmStages, 0, true}.smem(kSpmmStages);
+    const size_t smem =
+        StageLayout{((TW + 3) & ~3) * KC, P.trp_stride, false, kSpmmStages, 0, true}.smem(kSpmmStages);
+    CUtensorMap tmap;
+    const int use_tmap = (VEC == 4 && make_row_gather_map(&tmap, B, h->A.N, K, ldb, KC)) ? 1 : 0;
     if (P.n_dslots > 0 && P.dscratch_k < K) {
       SR_TRY(P.dscratch.alloc((size_t)P.n_dslots * P.panel_rows * K));
       P.dscratch_k = K;
@@ -782,7 +854,7 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
       kern<<<grid, (kDenseWarps + 1) * 32, smem, s>>>(
           P.units.p, (int)P.n_units, P.vtiles.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.dense_out.p, B, ldb, C, ldc,
           (int)K, TW, P.trp_stride, P.panel_rows, P.dscratch.p, P.dsplit_info.p, P.dsplit_counter.p, P.blobs.p,
-          P.blob_meta.p, flags);
+          P.blob_meta.p, tmap, use_tmap, flags);
       SR_CUDA_TRY(cudaGetLastError());
       return SR_OK;
     };
@@ -841,14 +913,16 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
   if (P.n_units > 0) {
     const int TW = P.tile_cols;
     const size_t smem =
-        StageLayout{TW * NCH_D * KC, P.trp_stride, true, kSddmmStages, 0, true}.smem(kSddmmStages);
+        StageLayout{((TW + 3) & ~3) * NCH_D * KC, P.trp_stride, true, kSddmmStages, 0, true}.smem(kSddmmStages);
+    CUtensorMap tmap;
+    const int use_tmap = (VEC == 4 && make_row_gather_map(&tmap, Y, h->A.N, K, ldy, NCH_D * KC)) ? 1 : 0;
     const unsigned grid = (unsigned)std::min<int64_t>(P.n_units, (int64_t)kDenseCtasPerSM * num_sms());
     const int flags = (VEC == 4 ? 1 : 0) | (dense_dbg() << 1);
     auto launch = [&](auto kern) -> int {
       SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
       kern<<<grid, (kDenseWarps + 1) * 32, smem, s>>>(
           P.units.p, (int)P.n_units, P.vtiles.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.d_oidx.p, P.pos_xrow.p, X, ldx,
-          Y, ldy, (int)K, TW, P.trp_stride, out, P.blobs.p, P.blob_meta.p, flags);
+          Y, ldy, (int)K, TW, P.trp_stride, out, P.blobs.p, P.blob_meta.p, tmap, use_tmap, flags);
       SR_CUDA_TRY(cudaGetLastError());
       return SR_OK;
     };
