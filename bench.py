@@ -301,8 +301,9 @@ def run_ours(args, A, ops, rank, world, local_rank):
     if dom and os.path.exists(prof_path):
         with open(prof_path) as f:
             tr = json.load(f)
-        key = f"{args.config}_K{K}_{dom}"
-        traffic = tr.get(key)
+        rec = tr.get(f"{args.config}_K{K}_{dom}")
+        if rec is not None and world == 1:
+            traffic = rec["bytes"]  # ncu --set full, per launch (profiles/ncu_traffic.py)
     roofline = None
     if dom:
         d = kern[dom]

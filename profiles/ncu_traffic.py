@@ -1,0 +1,40 @@
+"""Extract per-launch DRAM traffic (dram__bytes_read.sum + dram__bytes_write.sum) of libsr's
+kernels from an `ncu --set full ... --page raw --csv` export and merge it into
+profiles/ncu_traffic.json, keyed "<config>_K<K>_<kernel kind>" (bench.py reads it into the
+roofline `traffic` field).
+
+  python profiles/ncu_traffic.py <raw.csv> <config> <K> [source-tag]
+"""
+import csv
+import json
+import os
+import sys
+
+KINDS = {"spmm_dense_kernel": "spmm_dense_tiles", "spmm_sparse_kernel": "spmm_sparse_rows",
+         "sddmm_dense_kernel": "sddmm_dense_tiles", "sddmm_sparse_kernel": "sddmm_sparse_rows"}
+UNIT = {"byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
+
+
+def main(path, config, K, tag=""):
+    rows = list(csv.reader(open(path)))
+    hdr, units, data = rows[0], rows[1], rows[2:]
+    ix = {h: i for i, h in enumerate(hdr)}
+    out_path = os.path.join(os.path.dirname(os.path.abspath(__file__)), "ncu_traffic.json")
+    table = json.load(open(out_path)) if os.path.exists(out_path) else {}
+    for d in data:
+        name = d[ix["Kernel Name"]]
+        kind = next((v for k, v in KINDS.items() if k in name), None)
+        if kind is None:
+            continue
+        total = 0.0
+        for m in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
+            total += float(d[ix[m]]) * UNIT[units[ix[m]]]
+        t = float(d[ix["gpu__time_duration.sum"]]) * {"nsecond": 1e-9, "ns": 1e-9, "usecond": 1e-6, "us": 1e-6,
+                                                       "msecond": 1e-3, "ms": 1e-3}[units[ix["gpu__time_duration.sum"]]]
+        table[f"{config}_K{K}_{kind}"] = {"bytes": total, "ncu_duration_s": t, "source": tag or os.path.basename(path)}
+    json.dump(table, open(out_path, "w"), indent=1, sort_keys=True)
+    print(json.dumps(table, indent=1))
+
+
+if __name__ == "__main__":
+    main(*sys.argv[1:])
