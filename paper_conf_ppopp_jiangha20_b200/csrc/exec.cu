@@ -181,7 +181,16 @@ __global__ void __launch_bounds__(256, MINB) spmm_sparse_kernel(
       for (int k = lane * VEC; k < K; k += 32 * VEC) {
         Frag<VEC> s;
         s.zero();
-        for (int c = 0; c < si.y; ++c) {
+        int c = 0;
+        for (; c + 4 <= si.y; c += 4) {  // 4 partial loads in flight, summed in chunk order
+          Frag<VEC> p0, p1, p2, p3;
+          p0.load_cg(scratch + (int64_t)(si.x + c) * K + k);
+          p1.load_cg(scratch + (int64_t)(si.x + c + 1) * K + k);
+          p2.load_cg(scratch + (int64_t)(si.x + c + 2) * K + k);
+          p3.load_cg(scratch + (int64_t)(si.x + c + 3) * K + k);
+          s.add(p0); s.add(p1); s.add(p2); s.add(p3);
+        }
+        for (; c < si.y; ++c) {
           Frag<VEC> part;
           part.load_cg(scratch + (int64_t)(si.x + c) * K + k);
           s.add(part);
@@ -533,20 +542,33 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) spmm_
       if (threadIdx.x == 0) last_ticket = (atomicAdd(split_counter + si.x, 1) == si.y - 1);
       consumers_sync();
       if (last_ticket) {
+        // all 256 consumer threads share the (row, fragment) sums; chunk partials are added
+        // in chunk order with 4 loads in flight (a hub panel can have >100 chunks)
         __threadfence();
-        for (int i = 0; i < RPW; ++i) {
-          const int orow = __shfl_sync(FULL, out_row, i);
-          if (r0 + i >= hd.nrows || orow < 0) continue;
-          for (int k = lane * VEC; k < K; k += 32 * VEC) {
-            Frag<VEC> s;
-            s.zero();
-            for (int c = 0; c < si.y; ++c) {
-              Frag<VEC> part;
-              part.load_cg(scratch + ((int64_t)(si.x + c) * P + r0 + i) * K + k);
-              s.add(part);
-            }
-            s.store_cs(C + (int64_t)orow * ldc + k);
+        const int kq = (K + VEC - 1) / VEC;
+        for (int item = threadIdx.x; item < hd.nrows * kq; item += kDenseWarps * 32) {
+          const int r = item / kq, k = (item - r * kq) * VEC;
+          const int orow = dense_out[hd.q0 + r];
+          if (orow < 0) continue;
+          const float* src = scratch + ((int64_t)si.x * P + r) * K + k;
+          const int64_t cstride = (int64_t)P * K;
+          Frag<VEC> s;
+          s.zero();
+          int c = 0;
+          for (; c + 4 <= si.y; c += 4) {
+            Frag<VEC> p0, p1, p2, p3;
+            p0.load_cg(src + (c + 0) * cstride);
+            p1.load_cg(src + (c + 1) * cstride);
+            p2.load_cg(src + (c + 2) * cstride);
+            p3.load_cg(src + (c + 3) * cstride);
+            s.add(p0); s.add(p1); s.add(p2); s.add(p3);
           }
+          for (; c < si.y; ++c) {
+            Frag<VEC> p0;
+            p0.load_cg(src + c * cstride);
+            s.add(p0);
+          }
+          s.store_cs(C + (int64_t)orow * ldc + k);
         }
         consumers_sync();
         if (threadIdx.x == 0) split_counter[si.x] = 0;
