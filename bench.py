@@ -49,7 +49,10 @@ def parse():
     ap.add_argument("--panel-rows", type=int, default=64)
     ap.add_argument("--tile-cols", type=int, default=64)
     ap.add_argument("--max-bucket", type=int, default=32)
-    ap.add_argument("--dense-min", type=int, default=2)
+    # ASpT dense-column threshold (R17).  The paper's example is 2 (a P100 with 64 KB of
+    # shared memory per SM); on B200 (126 MB L2, 128-bit gathers at 8 CTAs/SM) staging pays only
+    # for columns shared by about half the panel: sweep in profiles/r01/NOTES.md.
+    ap.add_argument("--dense-min", type=int, default=32)
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target CPU work of cpu_baseline")
     ap.add_argument("--no-cpu-baseline", action="store_true")
