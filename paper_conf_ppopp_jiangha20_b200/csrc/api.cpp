@@ -102,45 +102,11 @@ void sparse_traffic(const ItemBuilder& ib, int64_t n_nonzero, int64_t n_zero, co
   t.sparse_distinct_cols = distinct;
 }
 
-// Streamed phase-S tasks: runs of consecutive items whose entries are contiguous in the
-// remainder stream (<= kTaskNnz entries, <= kTaskItems items); one lane group pipelines a
-// task's entries across its row boundaries.  Zero-row items form their own tasks at the end.
-constexpr int64_t kTaskNnz = 384, kTaskItems = 64;
-void build_tasks(const ItemBuilder& ib, int64_t n_nonzero, std::vector<int2>& tasks, int64_t* n_stasks) {
-  const int64_t n = (int64_t)ib.items.size();
-  tasks.clear();
-  int64_t i = 0;
-  while (i < n_nonzero) {
-    int64_t j = i, nnz = 0;
-    while (j < n_nonzero && nnz < kTaskNnz && j - i < kTaskItems) {
-      nnz += ib.items[j].e1 - ib.items[j].e0;
-      ++j;
-    }
-    tasks.push_back(make_int2((int)i, (int)j));
-    i = j;
-  }
-  *n_stasks = (int64_t)tasks.size();
-  for (; i < n; i += kTaskItems) tasks.push_back(make_int2((int)i, (int)std::min(n, i + kTaskItems)));
-}
-
-// The last entry of every non-empty item carries kEntLast in its column word: the streamed
-// phase-S kernels switch rows on that bit instead of comparing positions with row ends.
-void mark_item_ends(const ItemBuilder& ib, int64_t n_nonzero, std::vector<int2>& ent) {
-  for (int64_t i = 0; i < n_nonzero; ++i) {
-    const Item& x = ib.items[i];
-    if (x.e1 > x.e0) ent[x.e1 - 1].x |= (int32_t)kEntLast;
-  }
-}
-
 int upload_items(DevPlan& P, ItemBuilder& ib, int64_t n_sddmm_items, cudaStream_t s) {
   P.n_items = (int64_t)ib.items.size();
   P.n_sitems = n_sddmm_items;
   SR_TRY(P.items.upload(ib.items, s));
   SR_TRY(P.item_meta.upload(ib.meta, s));
-  std::vector<int2> tasks;
-  build_tasks(ib, n_sddmm_items, tasks, &P.n_stasks);
-  P.n_tasks = (int64_t)tasks.size();
-  SR_TRY(P.tasks.upload(tasks, s));
   P.n_slots = ib.n_slots;
   if (ib.n_slots > 0) {
     SR_TRY(P.split_info.upload(ib.split_info, s));
@@ -185,7 +151,6 @@ int build_identity_plan(sr_csr_s* h, cudaStream_t s) {
   }
   std::memset(&P.traffic, 0, sizeof(P.traffic));
   sparse_traffic(ib, n_nonzero, (int64_t)zero_rows.size(), ent, A.N, P.traffic);
-  mark_item_ends(ib, n_nonzero, ent);
   SR_TRY(P.s_ent.upload(ent, s));
   SR_TRY(upload_items(P, ib, n_nonzero, s));
   P.n_units = 0;
@@ -419,7 +384,6 @@ int build_exec_plan(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s) {
       tm.rmw_rows += d && r;
     }
   }
-  mark_item_ends(ib, n_nonzero, se);
   SR_TRY(P.s_ent.upload(se, s));
   SR_TRY(P.s_oidx.upload(so, s));
   SR_TRY(upload_items(P, ib, n_nonzero, s));

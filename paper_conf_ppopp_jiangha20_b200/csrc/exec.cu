@@ -141,7 +141,7 @@ __global__ void __launch_bounds__(256, MINB) spmm_sparse_kernel(
         for (int u = 0; u < U; ++u) {
           const int j = base + u * G + g;
           const int src = j & 31;
-          const int cf = __shfl_sync(FULL, my.x, src) & 0x7fffffff;  // drop kEntLast
+          const int cf = __shfl_sync(FULL, my.x, src);
           const float v = __int_as_float(__shfl_sync(FULL, my.y, src));
           const bool ok = (j < n) && kv;
           a[u] = ok ? v : 0.f;
@@ -235,7 +235,7 @@ __global__ void __launch_bounds__(256, MINB) sddmm_sparse_kernel(
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         const int j = base + u * G + g;
-        const int c = __shfl_sync(FULL, my.x, j & 31) & 0x7fffffff;  // drop kEntLast
+        const int c = __shfl_sync(FULL, my.x, j & 31);
         const bool ok = j < n;
         float d = 0.f;
 #pragma unroll
@@ -263,361 +263,6 @@ __global__ void __launch_bounds__(256, MINB) sddmm_sparse_kernel(
       }
     }
   }
-}
-
-// ------------------------------------------------------------------ phase S: streamed
-// One warp runs one task: a run of consecutive items (remainder rows in perm2 order, chunks
-// of long rows, or zero rows) whose entries are contiguous in the remainder stream.  The
-// task's gathered B/Y rows flow through a private shared-memory ring ACROSS row boundaries:
-// each row is one LDGSTS.128 per lane (cp.async, no register held while in flight) issued D
-// entries ahead of the arithmetic, in blocks of 8 entries (one commit group each).  A warp
-// thus keeps D rows in flight whatever the row lengths — the register-held gathers of the
-// row kernels above are bounded by the row (R-MAT remainder rows average ~10 nnz), which
-// left phase S latency-bound (profiles/r01/NOTES.md).  Entries (col, val) come in chunks of
-// 32 (one per lane, two chunks ahead in registers) and items in windows of 32 (one per lane,
-// next window prefetched), so neither a row switch nor an issue waits on a global load.
-__device__ __forceinline__ void cp_async16(void* s, const void* g) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(s)), "l"(g) : "memory");
-}
-__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_wait() {
-  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
-}
-
-constexpr int kStreamBS = 8;  // entries per pipeline block (one cp.async group)
-
-struct ItemCursor {
-  const Item* items;
-  const uint32_t* meta;
-  int t0, t1, it, lane;
-  Item w, wn;  // lane l: item (window base + l), next window
-  uint32_t m, mn;
-  Item cur;    // the current item (warp-uniform)
-  uint32_t cm;
-  __device__ __forceinline__ void load(int base, Item& x, uint32_t& mm) const {
-    const int i = base + lane;
-    if (i < t1) {
-      x = items[i];
-      mm = meta ? meta[i] : 0u;
-    } else {
-      x = Item{0, 0, 0, 0};
-      mm = 0u;
-    }
-  }
-  __device__ __forceinline__ void select() {
-    const int s = (it - t0) & 31;
-    cur.e1 = __shfl_sync(FULL, w.e1, s);
-    cur.xrow = __shfl_sync(FULL, w.xrow, s);
-    cur.out = __shfl_sync(FULL, w.out, s);
-    cm = __shfl_sync(FULL, m, s);
-  }
-  __device__ __forceinline__ void init(int a, int b) {
-    t0 = a;
-    t1 = b;
-    it = a;
-    load(a, w, m);
-    load(a + 32, wn, mn);
-    select();
-  }
-  __device__ __forceinline__ bool next() {
-    if (++it >= t1) return false;
-    if (((it - t0) & 31) == 0) {
-      w = wn;
-      m = mn;
-      load(it + 32, wn, mn);
-    }
-    select();
-    return true;
-  }
-  // X row of item it+1 (SDDMM prefetch), or -1
-  __device__ __forceinline__ int peek_xrow() const {
-    const int j = it + 1;
-    const int s = (j - t0) & 31;
-    const int a = __shfl_sync(FULL, w.xrow, s), b = __shfl_sync(FULL, wn.xrow, s);
-    if (j >= t1) return -1;
-    return (((j - t0) >> 5) == ((it - t0) >> 5)) ? a : b;
-  }
-};
-
-// Split long row: the last chunk to finish sums all chunk partials in chunk order
-// (deterministic) and writes (or read-modify-writes) the C row.  Rare: kept out of line.
-__device__ __noinline__ void spmm_split_combine(uint32_t mt, int out, int K, float* __restrict__ C, int64_t ldc,
-                                                const float* __restrict__ scratch,
-                                                const int2* __restrict__ split_info, int* __restrict__ split_counter) {
-  const int lane = threadIdx.x & 31;
-  __threadfence();
-  __syncwarp();
-  const int2 si = split_info[mt & kItemSlotMask];
-  int last = 0;
-  if (lane == 0) last = (atomicAdd(split_counter + si.x, 1) == si.y - 1);
-  last = __shfl_sync(FULL, last, 0);
-  if (!last) return;
-  __threadfence();
-  for (int k = lane * 4; k < K; k += 128) {
-    Frag<4> s;
-    s.zero();
-    int c = 0;
-    for (; c + 4 <= si.y; c += 4) {
-      Frag<4> p0, p1, p2, p3;
-      p0.load_cg(scratch + (int64_t)(si.x + c) * K + k);
-      p1.load_cg(scratch + (int64_t)(si.x + c + 1) * K + k);
-      p2.load_cg(scratch + (int64_t)(si.x + c + 2) * K + k);
-      p3.load_cg(scratch + (int64_t)(si.x + c + 3) * K + k);
-      s.add(p0); s.add(p1); s.add(p2); s.add(p3);
-    }
-    for (; c < si.y; ++c) {
-      Frag<4> p;
-      p.load_cg(scratch + (int64_t)(si.x + c) * K + k);
-      s.add(p);
-    }
-    float* dst = C + (int64_t)out * ldc + k;
-    if (mt & kItemRMW) {
-      Frag<4> old;
-      old.load_cg(dst);
-      s.add(old);
-    }
-    s.store_cs(dst);
-  }
-  if (lane == 0) split_counter[si.x] = 0;
-}
-
-// SpMM flush of the warp's finished item (row, or chunk of a split row).
-__device__ __forceinline__ void spmm_flush(Frag<4>& acc, const ItemCursor& ic, bool kv, bool last_pass, int kk, int K,
-                                           float* __restrict__ C, int64_t ldc, float* __restrict__ scratch,
-                                           const int2* __restrict__ split_info, int* __restrict__ split_counter) {
-  if (kv) {
-    if (ic.cm & kItemSplit) {
-      acc.store(scratch + (int64_t)(ic.cm & kItemSlotMask) * K + kk);
-    } else {
-      float* dst = C + (int64_t)ic.cur.out * ldc + kk;
-      if (ic.cm & kItemRMW) {
-        Frag<4> old;
-        old.load_cg(dst);
-        acc.add(old);
-      }
-      acc.store_cs(dst);
-    }
-  }
-  acc.zero();
-  if ((ic.cm & kItemSplit) && last_pass)
-    spmm_split_combine(ic.cm, ic.cur.out, K, C, ldc, scratch, split_info, split_counter);
-}
-
-// One warp per task (SpMM), 128 columns per pass.  NBLK blocks (D = 8·NBLK entries, <= 32)
-// in flight; ring of NBLK+1 blocks of 8 rows × 512 bytes.  Entries past the task end read
-// as (col 0, val 0, no flag): their copies and FMAs are harmless, so the hot loop carries no
-// bounds predicates.  A set kEntLast bit closes the current item.
-template <int NBLK, int WPC>
-__global__ void __launch_bounds__(WPC * 32, (NBLK == 2 ? 4 : NBLK == 3 ? 3 : 2)) spmm_stream_kernel(
-    const int2* __restrict__ tasks, int64_t n_tasks, const Item* __restrict__ items,
-    const uint32_t* __restrict__ meta, const int2* __restrict__ ent, const float* __restrict__ B, int64_t ldb,
-    float* __restrict__ C, int64_t ldc, int K, float* __restrict__ scratch, const int2* __restrict__ split_info,
-    int* __restrict__ split_counter) {
-  constexpr int BS = kStreamBS, NR = NBLK + 1;
-  static_assert(NBLK * BS <= 32, "issue distance must stay within the next entry chunk");
-  extern __shared__ __align__(128) char smem_raw[];
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  float* const ring = reinterpret_cast<float*>(smem_raw) + (size_t)wid * (NR * BS * 128) + lane * 4;
-  const int64_t task = (int64_t)blockIdx.x * WPC + wid;
-  if (task >= n_tasks) return;
-  const int2 tk = tasks[task];
-  ItemCursor ic;
-  ic.items = items;
-  ic.meta = meta;
-  ic.lane = lane;
-  const int es = __ldg(&items[tk.x].e0);
-  const int n = __ldg(&items[tk.y - 1].e1) - es;
-  const int nblk = (n + BS - 1) / BS;
-  auto chunk = [&](int k) {  // entry es + 32k + lane
-    const int i = 32 * k + lane;
-    return i < n ? __ldcs(ent + es + i) : make_int2(0, 0);
-  };
-  for (int k0 = 0; k0 < K; k0 += 128) {
-    const int kk = k0 + lane * 4;
-    const bool kv = kk < K;
-    const bool last_pass = k0 + 128 >= K;
-    const float* const Bk = B + (kv ? kk : 0);
-    int2 c0 = chunk(0), c1 = chunk(1), c2 = chunk(2);  // chunks k, k+1, k+2 of the consume position
-    // issue block b into ring block rb, columns from chunk register cs
-    auto issue = [&](int b, float* dst, int cs) {
-      const int o = (b * BS) & 31;
-#pragma unroll
-      for (int j = 0; j < BS; ++j) {
-        const int col = __shfl_sync(FULL, cs, o + j) & 0x7fffffff;
-        cp_async16(dst + j * 128, Bk + (int64_t)col * ldb);
-      }
-    };
-#pragma unroll
-    for (int b = 0; b < NBLK; ++b) {
-      if (b < nblk) issue(b, ring + b * (BS * 128), b * BS < 32 ? c0.x : c1.x);
-      cp_commit();
-    }
-    ic.init(tk.x, tk.y);
-    Frag<4> acc;
-    acc.zero();
-    float* rc = ring;                       // ring block being consumed
-    float* ri = ring + NBLK * (BS * 128);   // ring block being filled
-    float* const rend = ring + NR * (BS * 128);
-    for (int c = 0; c < nblk; ++c) {
-      if (c > 0 && (c & 3) == 0) {
-        c0 = c1;
-        c1 = c2;
-        c2 = chunk((c >> 2) + 2);
-      }
-      cp_wait<NBLK - 1>();  // block c has landed (each lane reads only its own copies)
-      {
-        const int ib = c + NBLK;
-        if (ib < nblk) issue(ib, ri, ((ib * BS) >> 5) == (c >> 2) ? c0.x : c1.x);
-        cp_commit();
-      }
-      const int o = (c * BS) & 31;
-#pragma unroll
-      for (int j = 0; j < BS; ++j) {
-        const int cw = __shfl_sync(FULL, c0.x, o + j);
-        const float v = __int_as_float(__shfl_sync(FULL, c0.y, o + j));
-        Frag<4> bv;
-        bv.load_s(rc + j * 128);
-        acc.fma(v, bv);
-        if (cw < 0) {  // kEntLast: the item ends here
-          spmm_flush(acc, ic, kv, last_pass, kk, K, C, ldc, scratch, split_info, split_counter);
-          ic.next();
-        }
-      }
-      rc += BS * 128;
-      if (rc == rend) rc = ring;
-      ri += BS * 128;
-      if (ri == rend) ri = ring;
-    }
-    cp_wait<0>();
-    // trailing items: the zero rows of a zero-row task (non-empty items were closed by kEntLast)
-    while (ic.it < ic.t1) {
-      spmm_flush(acc, ic, kv, last_pass, kk, K, C, ldc, scratch, split_info, split_counter);
-      ic.next();
-    }
-  }
-}
-
-// SDDMM over a warp's task, K <= 128 (lane owns X/Y columns [4·lane, 4·lane+4)).  Per block
-// of 8 entries each lane forms 8 partial dot products; one transpose-reduction (9 shuffles
-// instead of 8 × 5) leaves entry ((lane>>4)&1)·4 + ((lane>>3)&1)·2 + ((lane>>2)&1) summed
-// over the warp in every lane, and lanes with lane % 4 == 0 write the 8 results.
-template <int NBLK, int WPC>
-__global__ void __launch_bounds__(WPC * 32, (NBLK == 2 ? 4 : NBLK == 3 ? 3 : 2)) sddmm_stream_kernel(
-    const int2* __restrict__ tasks, int64_t n_tasks, const Item* __restrict__ items, const int2* __restrict__ ent,
-    const int32_t* __restrict__ oidx, const float* __restrict__ X, int64_t ldx, const float* __restrict__ Y,
-    int64_t ldy, int K, float* __restrict__ out) {
-  constexpr int BS = kStreamBS, NR = NBLK + 1;
-  static_assert(NBLK * BS <= 32, "issue distance must stay within the next entry chunk");
-  extern __shared__ __align__(128) char smem_raw[];
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  float* const ring = reinterpret_cast<float*>(smem_raw) + (size_t)wid * (NR * BS * 128) + lane * 4;
-  const int64_t task = (int64_t)blockIdx.x * WPC + wid;
-  if (task >= n_tasks) return;
-  const int2 tk = tasks[task];
-  ItemCursor ic;
-  ic.items = items;
-  ic.meta = nullptr;
-  ic.lane = lane;
-  const int es = __ldg(&items[tk.x].e0);
-  const int n = __ldg(&items[tk.y - 1].e1) - es;
-  const int nblk = (n + BS - 1) / BS;
-  const int kk = lane * 4;
-  const bool kv = kk < K;
-  auto chunk = [&](int k) {
-    const int i = 32 * k + lane;
-    return i < n ? __ldcs(ent + es + i) : make_int2(0, 0);
-  };
-  auto ochunk = [&](int k) {
-    const int i = 32 * k + lane;
-    return i < n ? __ldcs(oidx + es + i) : 0;
-  };
-  auto load_x = [&](int row, Frag<4>& x) {
-    if (row >= 0 && kv) x.load_g(X + (int64_t)row * ldx + kk); else x.zero();
-  };
-  const float* const Yk = Y + (kv ? kk : 0);
-  int2 c0 = chunk(0), c1 = chunk(1), c2 = chunk(2);
-  int o0 = ochunk(0), o1 = ochunk(1), o2 = ochunk(2);
-  auto issue = [&](int b, float* dst, int cs) {
-    const int o = (b * BS) & 31;
-#pragma unroll
-    for (int j = 0; j < BS; ++j) {
-      const int col = __shfl_sync(FULL, cs, o + j) & 0x7fffffff;
-      cp_async16(dst + j * 128, Yk + (int64_t)col * ldy);
-    }
-  };
-#pragma unroll
-  for (int b = 0; b < NBLK; ++b) {
-    if (b < nblk) issue(b, ring + b * (BS * 128), b * BS < 32 ? c0.x : c1.x);
-    cp_commit();
-  }
-  ic.init(tk.x, tk.y);
-  Frag<4> x, xn;
-  load_x(ic.cur.xrow, x);
-  load_x(ic.peek_xrow(), xn);
-  float* rc = ring;
-  float* ri = ring + NBLK * (BS * 128);
-  float* const rend = ring + NR * (BS * 128);
-  const int my_e = ((lane >> 4) & 1) * 4 + ((lane >> 3) & 1) * 2 + ((lane >> 2) & 1);
-  for (int c = 0; c < nblk; ++c) {
-    if (c > 0 && (c & 3) == 0) {
-      c0 = c1;
-      c1 = c2;
-      c2 = chunk((c >> 2) + 2);
-      o0 = o1;
-      o1 = o2;
-      o2 = ochunk((c >> 2) + 2);
-    }
-    cp_wait<NBLK - 1>();
-    {
-      const int ib = c + NBLK;
-      if (ib < nblk) issue(ib, ri, ((ib * BS) >> 5) == (c >> 2) ? c0.x : c1.x);
-      cp_commit();
-    }
-    const int o = (c * BS) & 31;
-    float p[BS];
-#pragma unroll
-    for (int j = 0; j < BS; ++j) {
-      const int cw = __shfl_sync(FULL, c0.x, o + j);
-      Frag<4> y;
-      y.load_s(rc + j * 128);
-      p[j] = x.dot(y);
-      if (cw < 0) {  // kEntLast: move to the next row's X fragment
-        if (ic.next()) {
-          x = xn;
-          load_x(ic.peek_xrow(), xn);
-        }
-      }
-    }
-    // transpose-reduce the 8 partial dot products over the warp
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      const bool up = lane & 16;
-      const float send = up ? p[i] : p[i + 4], keep = up ? p[i + 4] : p[i];
-      p[i] = keep + __shfl_xor_sync(FULL, send, 16);
-    }
-#pragma unroll
-    for (int i = 0; i < 2; ++i) {
-      const bool up = lane & 8;
-      const float send = up ? p[i] : p[i + 2], keep = up ? p[i + 2] : p[i];
-      p[i] = keep + __shfl_xor_sync(FULL, send, 8);
-    }
-    {
-      const bool up = lane & 4;
-      const float send = up ? p[0] : p[1], keep = up ? p[1] : p[0];
-      p[0] = keep + __shfl_xor_sync(FULL, send, 4);
-    }
-    p[0] += __shfl_xor_sync(FULL, p[0], 2);
-    p[0] += __shfl_xor_sync(FULL, p[0], 1);
-    const float v = __int_as_float(__shfl_sync(FULL, c0.y, o + my_e));
-    const int oi = __shfl_sync(FULL, o0, o + my_e);
-    if ((lane & 3) == 0 && c * BS + my_e < n) __stcs(out + oi, v * p[0]);
-    rc += BS * 128;
-    if (rc == rend) rc = ring;
-    ri += BS * 128;
-    if (ri == rend) ri = ring;
-  }
-  cp_wait<0>();
 }
 
 // ------------------------------------------------------------------ phase D
@@ -1196,41 +841,6 @@ int sparse_variant() {
   return v;
 }
 
-// Phase-S engine: streamed warp pipelines (default, K in (64, 128·n] for SpMM, (64, 128] for
-// SDDMM) or the row kernels (SR_STREAM=0).  SR_STREAM=<NBLK> sets the blocks of 8 rows in
-// flight per warp (2, 3 or 4).
-int stream_engine() {
-  static const int v = [] {
-    const char* d = getenv("SR_STREAM");
-    return d ? atoi(d) : 3;
-  }();
-  return v;
-}
-
-template <int NBLK, int WPC>
-int launch_spmm_stream(DevPlan& P, const float* B, int64_t ldb, float* C, int64_t ldc, int K, cudaStream_t s) {
-  const size_t smem = (size_t)WPC * (NBLK + 1) * kStreamBS * 128 * 4;
-  auto kern = spmm_stream_kernel<NBLK, WPC>;
-  SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  const unsigned grid = (unsigned)((P.n_tasks + WPC - 1) / WPC);
-  kern<<<grid, WPC * 32, smem, s>>>(P.tasks.p, P.n_tasks, P.items.p, P.item_meta.p, P.s_ent.p, B, ldb, C, ldc, K,
-                                    P.scratch.p, P.split_info.p, P.split_counter.p);
-  SR_CUDA_TRY(cudaGetLastError());
-  return SR_OK;
-}
-
-template <int NBLK, int WPC>
-int launch_sddmm_stream(DevPlan& P, const float* X, int64_t ldx, const float* Y, int64_t ldy, int K, float* out,
-                        cudaStream_t s) {
-  const size_t smem = (size_t)WPC * (NBLK + 1) * kStreamBS * 128 * 4;
-  auto kern = sddmm_stream_kernel<NBLK, WPC>;
-  SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  const unsigned grid = (unsigned)((P.n_stasks + WPC - 1) / WPC);
-  kern<<<grid, WPC * 32, smem, s>>>(P.tasks.p, P.n_stasks, P.items.p, P.s_ent.p, P.s_oidx.p, X, ldx, Y, ldy, K, out);
-  SR_CUDA_TRY(cudaGetLastError());
-  return SR_OK;
-}
-
 int num_sms() {
   static int n = 0;
   if (n == 0) {
@@ -1294,18 +904,8 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
       SR_TRY(P.scratch.alloc((size_t)P.n_slots * K));
       P.scratch_k = K;
     }
-    if (P.profiling) SR_TRY(prof_begin(P, 2, s));
-    if constexpr (VEC == 4 && LPG == 32) if (stream_engine() > 0) {
-      switch (stream_engine()) {
-        case 2: SR_TRY((launch_spmm_stream<2, 4>(P, B, ldb, C, ldc, (int)K, s))); break;
-        case 4: SR_TRY((launch_spmm_stream<4, 4>(P, B, ldb, C, ldc, (int)K, s))); break;
-        default: SR_TRY((launch_spmm_stream<3, 4>(P, B, ldb, C, ldc, (int)K, s))); break;
-      }
-      if (P.profiling) SR_TRY(prof_end(P, s));
-      ++*launches;
-      return SR_OK;
-    }
     const unsigned grid = (unsigned)((P.n_items + kSparseWarps - 1) / kSparseWarps);
+    if (P.profiling) SR_TRY(prof_begin(P, 2, s));
     auto go = [&](auto kern) {
       kern<<<grid, kSparseWarps * 32, 0, s>>>(P.items.p, P.item_meta.p, P.n_items, P.s_ent.p, B, ldb, C, ldc, (int)K,
                                                P.scratch.p, P.split_info.p, P.split_counter.p);
@@ -1356,18 +956,8 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
     ++*launches;
   }
   if (P.n_sitems > 0) {
-    if (P.profiling) SR_TRY(prof_begin(P, 4, s));
-    if constexpr (VEC == 4) if (K > 64 && K <= 128 && stream_engine() > 0) {
-      switch (stream_engine()) {
-        case 2: SR_TRY((launch_sddmm_stream<2, 4>(P, X, ldx, Y, ldy, (int)K, out, s))); break;
-        case 4: SR_TRY((launch_sddmm_stream<4, 4>(P, X, ldx, Y, ldy, (int)K, out, s))); break;
-        default: SR_TRY((launch_sddmm_stream<3, 4>(P, X, ldx, Y, ldy, (int)K, out, s))); break;
-      }
-      if (P.profiling) SR_TRY(prof_end(P, s));
-      ++*launches;
-      return SR_OK;
-    }
     const unsigned grid = (unsigned)((P.n_sitems + kSparseWarps - 1) / kSparseWarps);
+    if (P.profiling) SR_TRY(prof_begin(P, 4, s));
     auto go = [&](auto kern) {
       kern<<<grid, kSparseWarps * 32, 0, s>>>(P.items.p, P.n_sitems, P.s_ent.p, P.s_oidx.p, X, ldx, Y, ldy, (int)K,
                                                out);

@@ -99,7 +99,6 @@ struct __align__(16) Item {
   int32_t out;   // SpMM output row (original id, or packed shard index)
 };
 
-constexpr uint32_t kEntLast = 1u << 31;    // s_ent[e].x: entry e ends its item (column in the low 31 bits)
 constexpr uint32_t kItemRMW = 1u << 31;    // C[out] += partial (row also has dense-tile nnz)
 constexpr uint32_t kItemSplit = 1u << 30;  // partial of a split long row -> scratch slot
 constexpr uint32_t kItemSlotMask = (1u << 30) - 1;
@@ -156,8 +155,6 @@ struct DevPlan {
   int64_t n_items = 0;
   DevBuf<Item> sitems;        // SDDMM items (remainder rows / chunks only)
   int64_t n_sitems = 0;
-  DevBuf<int2> tasks;         // streamed phase S: item runs [t0, t1) (SDDMM: the first n_stasks)
-  int64_t n_tasks = 0, n_stasks = 0;
   DevBuf<int2> split_info;    // per scratch slot: {first slot, nchunks}
   DevBuf<int32_t> split_counter;
   int64_t n_slots = 0;
