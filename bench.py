@@ -214,6 +214,42 @@ def model_bytes(kind: str, tm: dict, K: int) -> float:
     return algorithmic_bytes(kind, tm, K) + row * (tm["dense_col_loads"] - tm["dense_distinct_cols"])
 
 
+def gathered_bytes(kind: str, tm: dict, K: int) -> float:
+    """Bytes the kernel moves from L2/HBM into the SMs for its gathered dense rows: one K·4-byte
+    row per remainder nnz (phase S), one per staged dense column of a tile (phase D)."""
+    row = 4.0 * K
+    return row * (tm["sparse_nnz"] if kind.endswith("sparse_rows") else tm["dense_col_loads"])
+
+
+def gather_ceiling(table_bytes: float, K: int):
+    """Measured random-row-gather bandwidth for a table of this size (profiles/gather_bw.cu,
+    committed results in profiles/r01/gather_bw.jsonl; 8 CTAs/SM series), log-interpolated in
+    the table size, nearest row width (128 or 512 bytes)."""
+    path = os.path.join(ROOT, "profiles", "r01", "gather_bw.jsonl")
+    if not os.path.exists(path):
+        return None, None
+    pts = []
+    rb = 512 if K * 4 >= 320 else 128
+    with open(path) as f:
+        for line in f:
+            d = json.loads(line)
+            if d.get("row_bytes") == rb and d.get("ctas_per_sm") == 8:
+                pts.append((d["table_MB"] * 2.0 ** 20, d["gather_GBs"]))
+    if not pts:
+        return None, None
+    pts.sort()
+    import math
+    x = min(max(table_bytes, pts[0][0]), pts[-1][0])
+    for (x0, y0), (x1, y1) in zip(pts, pts[1:]):
+        if x0 <= x <= x1:
+            w = (math.log(x) - math.log(x0)) / (math.log(x1) - math.log(x0)) if x1 > x0 else 0.0
+            y = y0 + w * (y1 - y0)
+            break
+    else:
+        y = pts[-1][1]
+    return y, f"profiles/r01/gather_bw.jsonl: random {rb}-byte row gathers, {table_bytes / 2**20:.0f} MB table (interpolated)"
+
+
 def run_ours(args, A, ops, rank, world, local_rank):
     import torch
     import paper_conf_ppopp_jiangha20_b200 as sr
@@ -314,6 +350,18 @@ def run_ours(args, A, ops, rank, world, local_rank):
                     "frac": d["achieved_gbs"] / peak, "traffic": traffic, "peak_source": peak_src,
                     "algorithmic_bytes_per_launch": d["algorithmic_bytes"], "avg_ms": d["avg_ms"]}
 
+    # the same kernel against the measured random-gather ceiling of its operand's size: the
+    # gathered rows come from L2/HBM at a rate set by the table size (profiles/r01/NOTES.md)
+    gather_roof = None
+    if dom:
+        d = kern[dom]
+        gb = gathered_bytes(dom, tm, K)
+        ceil_gbs, ceil_src = gather_ceiling(4.0 * K * A.ncols, K)
+        if ceil_gbs:
+            ach = gb / (d["avg_ms"] / 1e3) / 1e9
+            gather_roof = {"kernel": dom, "bound": "gather", "achieved": ach, "peak": ceil_gbs, "unit": "GB/s",
+                           "frac": ach / ceil_gbs, "gathered_bytes_per_launch": gb, "peak_source": ceil_src}
+
     # end to end through the public API with host buffers (pinned), per step
     e2e = None
     if args.e2e_steps > 0:
@@ -377,11 +425,14 @@ def run_ours(args, A, ops, rank, world, local_rank):
             "config": {"workload": f"{args.config} (configs[{list(gen.CONFIGS).index(args.config)}])",
                        "nrows": A.nrows, "ncols": A.ncols, "nnz": A.nnz, "K": K, "ops": ops,
                        "parallelism": f"row-panel shards x{world}" if world > 1 else "single GPU",
-                       "l2": "512 MB write between steps (outside timed intervals); B/X/Y > L2",
+                       "l2": "512 MB write between steps (outside timed intervals); "
+                             + ("B/X/Y larger than the 126 MB L2" if 4.0 * K * A.ncols > 126e6
+                                else "gathered operand fits the L2 (cold at each step start)"),
                        "plan": {"mode": args.mode, "panel_rows": args.panel_rows, "tile_cols": args.tile_cols,
                                 "max_bucket": args.max_bucket, "dense_min": args.dense_min, "siglen": 128, "bsize": 2, "threshold_size": 256,
                                 "seed": 4}},
             "roofline": roofline,
+            "gather_roofline": gather_roof,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": launches,

@@ -351,3 +351,20 @@ def test_dist_gather_single_rank_nccl(env, oracle):
         _sddmm_check(oracle, A, X.cpu().numpy(), Y.cpu().numpy(), out.cpu().numpy())
     finally:
         tdist.destroy_process_group()
+
+
+# ------------------------------------------------------------------ alternative phase-D engines
+@pytest.mark.parametrize("engine", ["coop", "l1"])
+def test_dense_engines_subprocess(env, engine):
+    """The phase-D engine is chosen once per process (SR_DENSE_ENGINE); rerun the numeric
+    parity cases that exercise dense tiles (K sweep incl. multi-pass K, tile widths, split
+    hub panels + RMW rows) under the non-default engines."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    e = dict(os.environ, SR_DENSE_ENGINE=engine)
+    r = subprocess.run([sys.executable, "-m", "pytest", os.path.join(root, "tests", "test_gpu_parity.py"), "-m", "gpu",
+                        "-q", "-x", "-p", "no:cacheprovider", "-k", "k_sweep or tile_widths or long_rows"],
+                       cwd=root, env=e, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
