@@ -288,7 +288,8 @@ def run_ours(args, A, ops, rank, world, local_rank):
                 M.sddmm(X, Y, out, stream=stream)
             ev[i][1].record(stream)
             n = M.last_launch_count()
-            times = M.last_kernel_times()  # waits for this op
+            times = M.last_kernel_times()  # waits for the library's own events of this op
+            ev[i][1].synchronize()
             total += ev[i][0].elapsed_time(ev[i][1])
             if record:
                 launches += n

@@ -2,6 +2,7 @@
 // decision rules P:265), plan construction, metadata export, host entry points.
 #include <algorithm>
 #include <chrono>
+#include <cstdlib>
 #include <cstring>
 #include <numeric>
 #include <string>
@@ -102,7 +103,60 @@ void sparse_traffic(const ItemBuilder& ib, int64_t n_nonzero, int64_t n_zero, co
   t.sparse_distinct_cols = distinct;
 }
 
+// Row-group tasks of the SpMM phase-S kernel (exec.cu: spmm_task_kernel): greedy runs of
+// consecutive items, at most 32 items and task_nnz entries (a longer item stands alone; a
+// split chunk always stands alone), whose items are contiguous in the entry stream; a task holds
+// either only non-empty rows or only zero rows.
+int32_t task_nnz() {
+  static const int32_t v = [] {
+    const char* e = getenv("SR_TASK_NNZ");
+    const int x = e ? atoi(e) : 128;  // measured best of 32/64/128/256 on C2 (profiles/r01/NOTES.md)
+    return x < 1 ? 1 : x;
+  }();
+  return v;
+}
+
+std::vector<int4> build_tasks(const ItemBuilder& ib, int64_t n, int64_t max_rows) {
+  std::vector<int4> tasks;
+  const int32_t T = task_nnz();
+  int64_t i = 0;
+  while (i < n) {
+    const int64_t start = i;
+    int32_t e0 = -1, e1 = -1;
+    if (ib.meta[i] & kItemSplit) {
+      e0 = ib.items[i].e0;
+      e1 = ib.items[i].e1;
+      ++i;
+    } else {
+      int32_t tot = 0;
+      const bool zero = ib.items[i].e1 == ib.items[i].e0;
+      while (i < n && i - start < max_rows && !(ib.meta[i] & kItemSplit)) {
+        const Item& x = ib.items[i];
+        const int32_t len = x.e1 - x.e0;
+        if ((len == 0) != zero) break;  // zero rows and non-empty rows go to separate tasks
+        if (len > 0) {
+          if (e0 >= 0 && (x.e0 != e1 || tot + len > T)) break;
+          if (e0 < 0) e0 = e1 = x.e0;
+          e1 += len;
+          tot += len;
+        }
+        ++i;
+      }
+      if (e0 < 0) e0 = e1 = 0;
+    }
+    tasks.push_back(make_int4(e0, e1, (int32_t)start, (int32_t)i));
+  }
+  return tasks;
+}
+
 int upload_items(DevPlan& P, ItemBuilder& ib, int64_t n_sddmm_items, cudaStream_t s) {
+  const std::vector<int4> tasks = build_tasks(ib, (int64_t)ib.items.size(), 32);
+  P.n_tasks = (int64_t)tasks.size();
+  SR_TRY(P.tasks.upload(tasks, s));
+  // SDDMM: the non-empty items only (a prefix), at most 8 rows per task (X rows staged in smem)
+  const std::vector<int4> stasks = build_tasks(ib, n_sddmm_items, 8);
+  P.n_stasks = (int64_t)stasks.size();
+  SR_TRY(P.stasks.upload(stasks, s));
   P.n_items = (int64_t)ib.items.size();
   P.n_sitems = n_sddmm_items;
   SR_TRY(P.items.upload(ib.items, s));

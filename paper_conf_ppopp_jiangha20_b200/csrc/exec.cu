@@ -122,10 +122,12 @@ __global__ void __launch_bounds__(256, MINB) spmm_sparse_kernel(
   constexpr int G = 32 / LPG;
   constexpr int KC = LPG * VEC;
   const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
-  const int64_t it = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const int64_t it = (int64_t)blockIdx.x * (blockDim.x >> 5) + __shfl_sync(FULL, threadIdx.x >> 5, 0);
   if (it >= n_items) return;
-  const Item item = items[it];
-  const uint32_t mt = meta[it];
+  Item item = items[it];  // warp-uniform through lane-0 shuffles (no divergent-shuffle fallback)
+  item.e0 = __shfl_sync(FULL, item.e0, 0); item.e1 = __shfl_sync(FULL, item.e1, 0);
+  item.xrow = __shfl_sync(FULL, item.xrow, 0); item.out = __shfl_sync(FULL, item.out, 0);
+  const uint32_t mt = __shfl_sync(FULL, meta[it], 0);
   for (int k0 = 0; k0 < K; k0 += KC) {
     const int kk = k0 + lg * VEC;
     const bool kv = kk < K;
@@ -217,9 +219,11 @@ __global__ void __launch_bounds__(256, MINB) sddmm_sparse_kernel(
   constexpr int G = 32 / LPG;
   constexpr int KC = LPG * VEC;
   const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
-  const int64_t it = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  const int64_t it = (int64_t)blockIdx.x * (blockDim.x >> 5) + __shfl_sync(FULL, threadIdx.x >> 5, 0);
   if (it >= n_items) return;
-  const Item item = items[it];
+  Item item = items[it];  // warp-uniform through lane-0 shuffles (no divergent-shuffle fallback)
+  item.e0 = __shfl_sync(FULL, item.e0, 0); item.e1 = __shfl_sync(FULL, item.e1, 0);
+  item.xrow = __shfl_sync(FULL, item.xrow, 0);
   Frag<VEC> x[NCH];
 #pragma unroll
   for (int c = 0; c < NCH; ++c) {
@@ -247,6 +251,251 @@ __global__ void __launch_bounds__(256, MINB) sddmm_sparse_kernel(
             d += x[ch].dot(y);
           }
         }
+        part[u] = d;
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+#pragma unroll
+        for (int off = LPG / 2; off > 0; off >>= 1) part[u] += __shfl_xor_sync(FULL, part[u], off);
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int j = base + u * G + g;
+        const float v = __int_as_float(__shfl_sync(FULL, my.y, j & 31));
+        const int o = __shfl_sync(FULL, myo, j & 31);
+        if (lg == 0 && j < n) __stcs(out + o, v * part[u]);
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------ phase S: SpMM, row-group tasks
+// One warp per task = up to 32 consecutive work items (rows in perm2 order, or zero rows) with
+// at most task_nnz entries, or one chunk of a split long row (api.cpp: build_tasks).  The warp
+// streams the task's entries with U row gathers in flight regardless of where rows end and
+// stores each row when its last entry has been added, so the per-row prologue of the one-row-
+// per-warp kernel (item descriptor -> entries -> first gather: two dependent latencies) is paid
+// once per task and short rows no longer limit the gathers in flight.  Each launch covers 128
+// columns (one float4 per lane; the host offsets B and C for K = 128·passes).  Rows are still
+// summed in CSR order, chunks of split rows combined in chunk order (deterministic).
+template <int U>
+__device__ __forceinline__ float4 task_row_sum(const int2* __restrict__ ent, int e0, int e1, const float* Bk,
+                                               uint32_t ldb, int lane) {
+  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int eb = e0; eb < e1; eb += 32) {
+    const int n = min(32, e1 - eb);
+    const int2 my = lane < n ? __ldcs(ent + eb + lane) : make_int2(0, 0);
+    for (int base = 0; base < n; base += U) {
+      float4 b[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        // past the end: re-load the last entry's row (same lines, no predicate, no zero fill)
+        const int c = __shfl_sync(FULL, my.x, min(base + u, n - 1));
+        b[u] = __ldg(reinterpret_cast<const float4*>(reinterpret_cast<const char*>(Bk) + (uint64_t)(uint32_t)c * ldb));
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const float a = __int_as_float(__shfl_sync(FULL, my.y, base + u));
+        if (base + u < n) {
+          acc.x = fmaf(a, b[u].x, acc.x); acc.y = fmaf(a, b[u].y, acc.y);
+          acc.z = fmaf(a, b[u].z, acc.z); acc.w = fmaf(a, b[u].w, acc.w);
+        }
+      }
+    }
+  }
+  return acc;
+}
+
+__device__ __forceinline__ void task_store(float4 v, uint32_t o, float* __restrict__ C, int64_t ldc, int lane) {
+  float4* dst = reinterpret_cast<float4*>(C + (int64_t)(o & 0x7fffffffu) * ldc) + lane;
+  if (o >> 31) {  // the row also has dense-tile entries (phase D ran first): read-modify-write
+    const float4 old = __ldcg(dst);
+    v.x += old.x; v.y += old.y; v.z += old.z; v.w += old.w;
+  }
+  __stcs(dst, v);
+}
+
+template <int U, int MINB>
+__global__ void __launch_bounds__(256, MINB) spmm_task_kernel(
+    const int4* __restrict__ tasks, int64_t n_tasks, const Item* __restrict__ items,
+    const uint32_t* __restrict__ meta, const int2* __restrict__ ent, const float* __restrict__ B, uint32_t ldb,
+    float* __restrict__ C, int64_t ldc, int K, int k0, float* __restrict__ scratch,
+    const int2* __restrict__ split_info, int* __restrict__ split_counter) {
+  const int lane = threadIdx.x & 31;
+  // warp-uniform values through lane-0 shuffles, so the compiler sees uniform control flow
+  // (no divergent-shuffle fallback paths and no stack frame)
+  const int64_t w = (int64_t)blockIdx.x * (blockDim.x >> 5) + __shfl_sync(FULL, threadIdx.x >> 5, 0);
+  if (w >= n_tasks) return;
+  int4 t = __ldg(tasks + w);  // {e0, e1, first item, end item}
+  t.x = __shfl_sync(FULL, t.x, 0); t.y = __shfl_sync(FULL, t.y, 0);
+  t.z = __shfl_sync(FULL, t.z, 0); t.w = __shfl_sync(FULL, t.w, 0);
+  const float* Bk = B + lane * 4;   // B, C are offset to this launch's 128 columns; ldb in bytes
+  const uint32_t m0 = __ldg(meta + t.z);
+  if (m0 & kItemSplit) {  // one chunk of a long row -> scratch; the last chunk combines in order
+    const float4 acc = task_row_sum<U>(ent, t.x, t.y, Bk, ldb, lane);
+    float* sc = scratch + k0 + lane * 4;
+    *reinterpret_cast<float4*>(sc + (int64_t)(m0 & kItemSlotMask) * K) = acc;
+    __threadfence();
+    __syncwarp();
+    const int2 si = __ldg(split_info + (m0 & kItemSlotMask));
+    int last = 0;
+    if (lane == 0) last = (atomicAdd(split_counter + si.x, 1) == si.y - 1);
+    last = __shfl_sync(FULL, last, 0);
+    if (!last) return;
+    __threadfence();
+    float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
+    int c = 0;
+    for (; c + 4 <= si.y; c += 4) {
+      float4 p[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) p[i] = __ldcg(reinterpret_cast<const float4*>(sc + (int64_t)(si.x + c + i) * K));
+#pragma unroll
+      for (int i = 0; i < 4; ++i) { s.x += p[i].x; s.y += p[i].y; s.z += p[i].z; s.w += p[i].w; }
+    }
+    for (; c < si.y; ++c) {
+      const float4 p = __ldcg(reinterpret_cast<const float4*>(sc + (int64_t)(si.x + c) * K));
+      s.x += p.x; s.y += p.y; s.z += p.z; s.w += p.w;
+    }
+    const int o = __ldg(reinterpret_cast<const int4*>(items) + t.z).w;
+    task_store(s, (uint32_t)o | ((m0 & kItemRMW) ? 0x80000000u : 0u), C, ldc, lane);
+    if (lane == 0) split_counter[si.x] = 0;
+    return;
+  }
+  const int cnt = t.w - t.z;
+  int end = 0;
+  uint32_t o = 0;  // output row | RMW flag in bit 31
+  if (lane < cnt) {
+    const int4 it = __ldg(reinterpret_cast<const int4*>(items) + t.z + lane);
+    end = it.y - it.x;
+    o = (uint32_t)it.w | ((__ldg(meta + t.z + lane) & kItemRMW) ? 0x80000000u : 0u);
+  }
+  if (t.x == t.y) {  // zero rows (build_tasks never mixes them with non-empty rows)
+    for (int r = 0; r < cnt; ++r) task_store(make_float4(0.f, 0.f, 0.f, 0.f), __shfl_sync(FULL, o, r), C, ldc, lane);
+    return;
+  }
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {  // inclusive scan: end of row r relative to the task's e0
+    const int v = __shfl_up_sync(FULL, end, d);
+    if (lane >= d) end += v;
+  }
+  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+  int r = 0;
+  int row_end = t.x + __shfl_sync(FULL, end, 0);
+  for (int eb = t.x; eb < t.y; eb += 32) {
+    const int n = min(32, t.y - eb);
+    const int2 my = lane < n ? __ldcs(ent + eb + lane) : make_int2(0, 0);
+    for (int base = 0; base < n; base += U) {
+      float4 b[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        // past the end: re-load the last entry's row (same lines, no predicate, no zero fill)
+        const int c = __shfl_sync(FULL, my.x, min(base + u, n - 1));
+        b[u] = __ldg(reinterpret_cast<const float4*>(reinterpret_cast<const char*>(Bk) + (uint64_t)(uint32_t)c * ldb));
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const float a = __int_as_float(__shfl_sync(FULL, my.y, base + u));
+        if (base + u < n) {
+          acc.x = fmaf(a, b[u].x, acc.x); acc.y = fmaf(a, b[u].y, acc.y);
+          acc.z = fmaf(a, b[u].z, acc.z); acc.w = fmaf(a, b[u].w, acc.w);
+          if (eb + base + u + 1 == row_end) {  // row r is complete (rows here are non-empty)
+            task_store(acc, __shfl_sync(FULL, o, r), C, ldc, lane);
+            acc = make_float4(0.f, 0.f, 0.f, 0.f);
+            ++r;
+            row_end = t.x + __shfl_sync(FULL, end, r & 31);
+          }
+        }
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------ phase S: SDDMM, row-group tasks
+// One warp per task = up to kSddmmTaskRows consecutive remainder rows (or one chunk of a long
+// row) with at most task_nnz entries.  At task start the lanes copy the task's X rows into the
+// warp's shared-memory slots with cp.async (in parallel with the entry load), so the stream of
+// Y gathers never waits on a per-row X load.  Geometry as sddmm_sparse_kernel: 8 lanes × NCH
+// float4 per nnz (K = 32·NCH), G = 4 nnz per warp step, U steps of gathers in flight; a group
+// whose next entry belongs to another row reloads its X fragment from shared memory.
+constexpr int kSddmmTaskRows = 8;
+
+__device__ __forceinline__ void cp_async_cg16(void* dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+
+template <int NCH, int U, int MINB>
+__global__ void __launch_bounds__(256, MINB) sddmm_task_kernel(
+    const int4* __restrict__ tasks, int64_t n_tasks, const Item* __restrict__ items, const int2* __restrict__ ent,
+    const int32_t* __restrict__ oidx, const float* __restrict__ X, int64_t ldx, const float* __restrict__ Y,
+    uint32_t ldy_bytes, float* __restrict__ out) {
+  constexpr int G = 4, LPG = 8;
+  __shared__ float4 xs[8][kSddmmTaskRows][NCH * 8];
+  const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
+  const int wid = __shfl_sync(FULL, threadIdx.x >> 5, 0);
+  const int64_t w = (int64_t)blockIdx.x * (blockDim.x >> 5) + wid;
+  if (w >= n_tasks) return;
+  int4 t = __ldg(tasks + w);  // {e0, e1, first item, end item}; warp-uniform via lane-0 shuffles
+  t.x = __shfl_sync(FULL, t.x, 0); t.y = __shfl_sync(FULL, t.y, 0);
+  t.z = __shfl_sync(FULL, t.z, 0); t.w = __shfl_sync(FULL, t.w, 0);
+  const int cnt = t.w - t.z;
+  int end = 0, xrow = 0;
+  if (lane < cnt) {
+    const int4 it = __ldg(reinterpret_cast<const int4*>(items) + t.z + lane);
+    end = it.y - it.x;
+    xrow = it.z;
+  }
+#pragma unroll
+  for (int d = 1; d < kSddmmTaskRows; d <<= 1) {  // inclusive scan over the (<= 8) rows
+    const int v = __shfl_up_sync(FULL, end, d);
+    if (lane >= d) end += v;
+  }
+  for (int r = 0; r < cnt; ++r) {  // stage the task's X rows (K·4 bytes each) in shared memory
+    const int xr = __shfl_sync(FULL, xrow, r);
+    if (lane < NCH * 8) cp_async_cg16(&xs[wid][r][lane], X + (int64_t)xr * ldx + lane * 4);
+  }
+  asm volatile("cp.async.commit_group;" ::: "memory");
+  const char* Yl = reinterpret_cast<const char*>(Y + lg * 4);
+  float4 x[NCH];
+  int cur = -1;
+  bool staged = false;
+  for (int eb = t.x; eb < t.y; eb += 32) {
+    const int n = min(32, t.y - eb);
+    const int2 my = lane < n ? __ldcs(ent + eb + lane) : make_int2(0, 0);
+    const int myo = lane < n ? __ldcs(oidx + eb + lane) : 0;
+    // row (within the task) of the entry this lane loaded
+    const int rel = eb + lane - t.x;
+    int myrow = 0;
+    for (int r = 0; r < cnt; ++r) myrow += (__shfl_sync(FULL, end, r) <= rel) ? 1 : 0;
+    if (!staged) {
+      cp_async_wait_all();
+      __syncwarp();
+      staged = true;
+    }
+    for (int base = 0; base < n; base += G * U) {
+      float4 y[U][NCH];
+      int row[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int jj = min(base + u * G + g, n - 1);
+        const int c = __shfl_sync(FULL, my.x, jj);
+        row[u] = __shfl_sync(FULL, myrow, jj);
+        const char* yp = Yl + (uint64_t)(uint32_t)c * ldy_bytes;
+#pragma unroll
+        for (int ch = 0; ch < NCH; ++ch) y[u][ch] = __ldg(reinterpret_cast<const float4*>(yp + ch * 128));
+      }
+      float part[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (row[u] != cur) {
+          cur = row[u];
+#pragma unroll
+          for (int ch = 0; ch < NCH; ++ch) x[ch] = xs[wid][cur][ch * 8 + lg];
+        }
+        float d = 0.f;
+#pragma unroll
+        for (int ch = 0; ch < NCH; ++ch)
+          d += fmaf(x[ch].x, y[u][ch].x, fmaf(x[ch].y, y[u][ch].y, fmaf(x[ch].z, y[u][ch].z, x[ch].w * y[u][ch].w)));
         part[u] = d;
       }
 #pragma unroll
@@ -1114,10 +1363,14 @@ int dense_engine() {  // 0 = coop, 1 = l1, 2 = tma
   return v;
 }
 
+// Phase-S kernel choice (SR_SPARSE_VARIANT, measurement knob; profiles/r01/NOTES.md):
+// default = row-group task kernels (SpMM U 4 at 8 CTAs/SM, SDDMM U 2 at 4 CTAs/SM);
+// 0 = one-row-per-warp kernels (U 2 / 8 CTAs); 1, 3 = row kernels at other occupancy points;
+// 4-7 = task kernels at other (U, CTAs/SM) points.
 int sparse_variant() {
   static const int v = [] {
     const char* d = getenv("SR_SPARSE_VARIANT");
-    return d ? atoi(d) : 0;
+    return d ? atoi(d) : 7;
   }();
   return v;
 }
@@ -1199,6 +1452,26 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
     }
     const unsigned grid = (unsigned)((P.n_items + kSparseWarps - 1) / kSparseWarps);
     if (P.profiling) SR_TRY(prof_begin(P, 2, s));
+    const int var = sparse_variant();
+    if (LPG == 32 && VEC == 4 && K % 128 == 0 && ldb * 4 < (1ll << 32) && var >= 4 && var <= 7 && P.n_tasks > 0) {
+      const unsigned tgrid = (unsigned)((P.n_tasks + kSparseWarps - 1) / kSparseWarps);
+      auto tk = [&](auto kern) {
+        for (int k0 = 0; k0 < K; k0 += 128)
+          kern<<<tgrid, kSparseWarps * 32, 0, s>>>(P.tasks.p, P.n_tasks, P.items.p, P.item_meta.p, P.s_ent.p,
+                                                    B + k0, (uint32_t)(ldb * 4), C + k0, ldc, (int)K, k0, P.scratch.p,
+                                                    P.split_info.p, P.split_counter.p);
+      };
+      switch (var) {
+        case 4: tk(spmm_task_kernel<4, 6>); break;
+        case 5: tk(spmm_task_kernel<8, 4>); break;
+        case 6: tk(spmm_task_kernel<2, 8>); break;
+        default: tk(spmm_task_kernel<4, 8>); break;
+      }
+      SR_CUDA_TRY(cudaGetLastError());
+      if (P.profiling) SR_TRY(prof_end(P, s));
+      ++*launches;
+      return SR_OK;
+    }
     auto go = [&](auto kern) {
       kern<<<grid, kSparseWarps * 32, 0, s>>>(P.items.p, P.item_meta.p, P.n_items, P.s_ent.p, B, ldb, C, ldc, (int)K,
                                                P.scratch.p, P.split_info.p, P.split_counter.p);
@@ -1263,6 +1536,26 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
   if (P.n_sitems > 0) {
     const unsigned grid = (unsigned)((P.n_sitems + kSparseWarps - 1) / kSparseWarps);
     if (P.profiling) SR_TRY(prof_begin(P, 4, s));
+    const int var = sparse_variant();
+    if (LPG == 8 && VEC == 4 && NCH <= 4 && K == 32 * NCH && ldy * 4 < (1ll << 32) && var >= 4 && var <= 7 &&
+        P.n_stasks > 0) {
+      const unsigned tgrid = (unsigned)((P.n_stasks + kSparseWarps - 1) / kSparseWarps);
+      auto tk = [&](auto kern) {
+        kern<<<tgrid, kSparseWarps * 32, 0, s>>>(P.stasks.p, P.n_stasks, P.items.p, P.s_ent.p, P.s_oidx.p, X, ldx,
+                                                  Y, (uint32_t)(ldy * 4), out);
+      };
+      constexpr int NC = NCH > 4 ? 4 : NCH;  // (NCH <= 4 guarded above; keeps NCH 8 instantiable)
+      switch (var) {
+        case 4: tk(sddmm_task_kernel<NC, 2, 4>); break;
+        case 5: tk(sddmm_task_kernel<NC, 1, 6>); break;
+        case 6: tk(sddmm_task_kernel<NC, 1, 5>); break;
+        default: tk(sddmm_task_kernel<NC, 2, 4>); break;
+      }
+      SR_CUDA_TRY(cudaGetLastError());
+      if (P.profiling) SR_TRY(prof_end(P, s));
+      ++*launches;
+      return SR_OK;
+    }
     auto go = [&](auto kern) {
       kern<<<grid, kSparseWarps * 32, 0, s>>>(P.items.p, P.n_sitems, P.s_ent.p, P.s_oidx.p, X, ldx, Y, ldy, (int)K,
                                                out);

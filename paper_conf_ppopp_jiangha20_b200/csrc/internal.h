@@ -153,6 +153,10 @@ struct DevPlan {
   DevBuf<Item> items;         // SpMM items (remainder rows, split chunks, zero rows)
   DevBuf<uint32_t> item_meta;
   int64_t n_items = 0;
+  DevBuf<int4> tasks;         // SpMM row-group tasks {e0, e1, first item, end item} (build_tasks)
+  int64_t n_tasks = 0;
+  DevBuf<int4> stasks;        // SDDMM row-group tasks (<= 8 rows each, non-empty rows only)
+  int64_t n_stasks = 0;
   DevBuf<Item> sitems;        // SDDMM items (remainder rows / chunks only)
   int64_t n_sitems = 0;
   DevBuf<int2> split_info;    // per scratch slot: {first slot, nchunks}

@@ -11,7 +11,8 @@ import os
 import sys
 
 KINDS = {"spmm_dense_kernel": "spmm_dense_tiles", "spmm_sparse_kernel": "spmm_sparse_rows",
-         "sddmm_dense_kernel": "sddmm_dense_tiles", "sddmm_sparse_kernel": "sddmm_sparse_rows"}
+         "spmm_task_kernel": "spmm_sparse_rows", "sddmm_dense_kernel": "sddmm_dense_tiles",
+         "sddmm_sparse_kernel": "sddmm_sparse_rows", "sddmm_task_kernel": "sddmm_sparse_rows"}
 UNIT = {"byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
 
 

@@ -11,4 +11,4 @@ timeout 600 python bench.py --K 32 > gpurun_out/${tag}_bench_k32.json 2> gpurun_
 timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/${tag}_bench_ref.json 2> gpurun_out/${tag}_bench_ref.err; echo "ref rc=$?"
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${tag}_launches.csv \
   python bench.py --steps 2 --warmup 1 --min-warm-s 0 --e2e-steps 0 --no-cpu-baseline > /dev/null 2>&1; echo "launches rc=$?"
-timeout 900 bash profiles/ncu_capture.sh ${tag}k128 "spmm_sparse|sddmm_sparse|spmm_dense|sddmm_dense" 4 > /dev/null 2>&1; echo "ncu k128 rc=$?"
+timeout 900 bash profiles/ncu_capture.sh ${tag}k128 "spmm_task|sddmm_task|spmm_dense|sddmm_dense" 4 > /dev/null 2>&1; echo "ncu k128 rc=$?"

@@ -148,7 +148,7 @@ def test_long_rows_split_and_rmw(env, oracle):
     rowptr, colidx = g._from_coo(n, m, np.concatenate(rows), np.concatenate(cols))
     A = g.CSR(n, m, rowptr, colidx, g._uniform_vals(colidx.size, 3))
     for params in (None, sr.default_params(**_plan_kw(16, 1, 8)), sr.default_params(**_plan_kw(16, 2, 0))):
-        for K in (32, 128):
+        for K in (32, 128, 256):  # 256: two 128-column passes of the SpMM task kernel
             M, B, X, Y, C, out = _run(env, A, K, params)
             _spmm_check(oracle, A, B, C)
             _sddmm_check(oracle, A, X, Y, out)
@@ -281,8 +281,8 @@ def test_full_size_sampled(env, oracle, config):
     plus the 20 longest rows (K=128, and K=32 for C2); SDDMM on every nnz of those rows."""
     sr, torch = env
     A = g.make(config)
-    kw = dict(siglen=128, bsize=2, seed=4, max_bucket=32, threshold_size=256, panel_rows=64, dense_min=2,
-              mode=0)
+    kw = dict(siglen=128, bsize=2, seed=4, max_bucket=32, threshold_size=256, panel_rows=64,
+              dense_min=32, mode=0)  # bench.py's plan (dense_min 32: profiles/r01/NOTES.md)
     M = sr.SparseMatrix.from_csr(A)
     M.reorder(sr.default_params(**kw))
     ref = oracle.plan(A, **kw)
@@ -353,17 +353,21 @@ def test_dist_gather_single_rank_nccl(env, oracle):
         tdist.destroy_process_group()
 
 
-# ------------------------------------------------------------------ alternative phase-D engines
-@pytest.mark.parametrize("engine", ["coop", "l1"])
-def test_dense_engines_subprocess(env, engine):
-    """The phase-D engine is chosen once per process (SR_DENSE_ENGINE); rerun the numeric
-    parity cases that exercise dense tiles (K sweep incl. multi-pass K, tile widths, split
-    hub panels + RMW rows) under the non-default engines."""
+# ------------------------------------------------------------------ alternative engines
+@pytest.mark.parametrize("var,val", [("SR_DENSE_ENGINE", "coop"), ("SR_DENSE_ENGINE", "l1"),
+                                     ("SR_SPARSE_VARIANT", "0"), ("SR_SPARSE_VARIANT", "5"),
+                                     ("SR_TASK_NNZ", "1")])
+def test_engines_subprocess(env, var, val):
+    """The phase-D engine (SR_DENSE_ENGINE) and the phase-S kernels (SR_SPARSE_VARIANT: 0 =
+    one-row-per-warp kernels, 5 = task kernels at another occupancy point; SR_TASK_NNZ=1 = one
+    row per task) are chosen once per process; rerun the numeric parity cases that exercise
+    them (K sweep incl. multi-pass K, tile widths, split rows + RMW rows) under the
+    non-default choices."""
     import os
     import subprocess
     import sys
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    e = dict(os.environ, SR_DENSE_ENGINE=engine)
+    e = dict(os.environ, **{var: val})
     r = subprocess.run([sys.executable, "-m", "pytest", os.path.join(root, "tests", "test_gpu_parity.py"), "-m", "gpu",
                         "-q", "-x", "-p", "no:cacheprovider", "-k", "k_sweep or tile_widths or long_rows"],
                        cwd=root, env=e, capture_output=True, text=True, timeout=900)
