@@ -117,8 +117,63 @@ int sr_spmm(sr_csr h, const float* B, int64_t K, int64_t ldb, float* C, int64_t 
 int sr_sddmm(sr_csr h, const float* X, int64_t ldx, const float* Y, int64_t ldy, int64_t K,
              float* out, sr_stream stream);
 
+/* -----------------------------------------------------------------------------
+ * sr_set_values — replace the nonzero values the kernels use; pattern and plan unchanged.
+ *   For iterative applications that reuse one plan with changing values, e.g. the
+ *   collaborative-filtering gradient loop: E := SDDMM(U, V) − R on the
+ *   pattern, then E·V with the same plan.
+ *   vals : DEVICE fp32 in the handle's OUTPUT order (the order sr_sddmm writes):
+ *          world == 1: [nnz], the caller's original nnz order; world > 1: [sr_shard_nnz],
+ *          this shard's packed order.
+ *   The device plan keeps the new values until the next sr_set_values; a later sr_reorder /
+ *   sr_plan_load rebuilds the plan from the values given to sr_csr_create.
+ * Asynchronous on `stream` (the caller keeps `vals` alive until it completes).
+ * Errors: SR_EINVAL, SR_ECUDA.
+ * ---------------------------------------------------------------------------*/
+int sr_set_values(sr_csr h, const float* vals, sr_stream stream);
+
 /* Free all host and device state.  NULL-safe.  Synchronises the device. */
 int sr_destroy(sr_csr h);
+
+/* -----------------------------------------------------------------------------
+ * Offline reordering ("data reordering can be performed offline", the
+ * preprocessing "amortized across iterations"): a plan is fully determined by the matrix,
+ * the parameters and the two row orders, so it can be saved once and loaded later without
+ * LSH or clustering (the tiling and the execution plan are rebuilt from perm1 / perm2).
+ *
+ * sr_plan_save — canonical byte image of h's plan into the HOST buffer buf[cap]:
+ *   "SRPLAN01" | u32 version 1 | u32 reserved | i64 M, N, nnz | u64 matrix fingerprint
+ *   (64-bit hash of the canonical rowptr / colidx) | sr_reorder_params | sr_plan_stats |
+ *   i64 len1, i32 perm1[len1] | i64 len2, i32 perm2[len2] | u64 checksum of all preceding
+ *   bytes.  *len gets the image size; buf may be NULL (size query).  The image does not
+ *   depend on world / rank (perm2 is global; a shard filters it).
+ *   Errors: SR_ESTATE (no plan: sr_reorder / sr_plan_load not called), SR_EINVAL (cap).
+ * sr_plan_load — install a saved plan on a handle of the SAME matrix (fingerprint checked)
+ *   that has no plan yet; world / rank select the shard (1, 0 = single GPU).  Synchronous.
+ *   Errors: SR_EINVAL (bad / corrupted image, other matrix, bad permutation, bad world /
+ *   rank), SR_ESTATE (the handle already has a plan), SR_ENOMEM, SR_ECUDA.
+ * ---------------------------------------------------------------------------*/
+int sr_plan_save(sr_csr h, void* buf, int64_t cap, int64_t* len);
+int sr_plan_load(sr_csr h, const void* buf, int64_t len, int32_t world, int32_t rank, sr_stream stream);
+
+/* -----------------------------------------------------------------------------
+ * sr_trial — trial-and-error plan selection ("perform row-reordering in the first
+ *   iteration and do SpMM or SDDMM on both the reordered matrix and the original matrix. If
+ *   the reordered matrix is faster, keep the row-reordering").  Times op (SR_OP_SPMM:
+ *   C := A·B with U = B, V unused, out = C; SR_OP_SDDMM: out := A ⊙ (U·Vᵀ) with U = X, V = Y)
+ *   `reps` times on each of the n candidate handles (plans of the same matrix: equal
+ *   nrows / ncols / nnz and shard output sizes, e.g. a reordered handle and a fresh one in the
+ *   original order) after one warm-up call each, on `stream` with CUDA events.  ms[i] gets the
+ *   median device time of candidate i (HOST array of n floats, may be NULL); *best the index
+ *   of the fastest.  Operands are DEVICE memory as in sr_spmm / sr_sddmm; `out` holds the last
+ *   candidate's result on return.  Synchronous.  Errors: SR_EINVAL (n < 1, NULL, candidates
+ *   of different shapes, reps < 1, bad op), SR_ECUDA.
+ * ---------------------------------------------------------------------------*/
+#define SR_OP_SPMM 0
+#define SR_OP_SDDMM 1
+int sr_trial(const sr_csr* cands, int32_t n, int32_t op, const float* U, int64_t ldu, const float* V,
+             int64_t ldv, int64_t K, float* out, int64_t ldo, int32_t reps, sr_stream stream, int32_t* best,
+             float* ms);
 
 /* ---------------------------------------------------------------------------
  * Plan metadata (bit-exact parity with the oracle; the gather/scatter step).

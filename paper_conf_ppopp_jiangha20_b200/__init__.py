@@ -18,6 +18,7 @@ LIB_PATH = os.path.join(_HERE, "libsr.so")
 
 SR_OK, SR_EINVAL, SR_ENOMEM, SR_ECUDA, SR_ESTATE, SR_EUNSUPPORTED = 0, -1, -2, -3, -4, -5
 AUTO, FORCE, OFF = 0, 1, 2
+SR_OP_SPMM, SR_OP_SDDMM = 0, 1
 
 
 class SRError(RuntimeError):
@@ -64,7 +65,7 @@ EXPORTED = ("sr_csr_create", "sr_default_params", "sr_reorder", "sr_spmm", "sr_s
             "sr_get_perm", "sr_get_plan_stats", "sr_export_tiles", "sr_shard_rows", "sr_shard_nnz_ids",
             "sr_last_launch_count", "sr_last_error", "sr_host_cluster", "sr_host_partition", "sr_version",
             "sr_get_traffic_model", "sr_set_profiling", "sr_last_kernel_times", "sr_scatter_rows",
-            "sr_scatter_values")
+            "sr_scatter_values", "sr_plan_save", "sr_plan_load", "sr_trial", "sr_set_values")
 
 _lib = None
 
@@ -100,6 +101,10 @@ def lib():
         "sr_last_kernel_times": (C.c_int, [P, P, P, i32, C.POINTER(i32)]),
         "sr_scatter_rows": (C.c_int, [P, i64, P, i64, i64, P, i64, P]),
         "sr_scatter_values": (C.c_int, [P, P, i64, P, P]),
+        "sr_plan_save": (C.c_int, [P, P, i64, C.POINTER(i64)]),
+        "sr_set_values": (C.c_int, [P, P, P]),
+        "sr_plan_load": (C.c_int, [P, P, i64, i32, i32, P]),
+        "sr_trial": (C.c_int, [P, i32, i32, P, i64, P, i64, i64, P, i64, i32, P, C.POINTER(i32), P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -183,6 +188,25 @@ class SparseMatrix:
         p = params if params is not None else default_params(**overrides)
         s = C.c_void_p(int(stream.cuda_stream)) if stream is not None else C.c_void_p()
         _check(lib().sr_reorder(self._h, C.byref(p), s))
+        self.params = p
+        return self.stats()
+
+    def save_plan(self) -> bytes:
+        """Canonical byte image of the plan (sr_plan_save: offline reordering)."""
+        n = C.c_int64()
+        _check(lib().sr_plan_save(self._h, None, 0, C.byref(n)))
+        buf = C.create_string_buffer(n.value)
+        _check(lib().sr_plan_save(self._h, C.cast(buf, C.c_void_p), n.value, C.byref(n)))
+        return buf.raw[:n.value]
+
+    def load_plan(self, image: bytes, world: int = 1, rank: int = 0, stream=None) -> dict:
+        """Install a saved plan of this matrix (sr_plan_load; no LSH / clustering)."""
+        s = C.c_void_p(int(stream.cuda_stream)) if stream is not None else C.c_void_p()
+        buf = C.create_string_buffer(bytes(image), len(image))
+        _check(lib().sr_plan_load(self._h, C.cast(buf, C.c_void_p), len(image), world, rank, s))
+        p = ReorderParams()
+        lib().sr_default_params(C.byref(p))
+        p.world, p.rank = world, rank
         self.params = p
         return self.stats()
 
@@ -270,6 +294,14 @@ class SparseMatrix:
         _check(lib().sr_spmm(self._h, _ptr(B), K, B.stride(0), _ptr(C_out), C_out.stride(0), _stream(stream)))
         return C_out
 
+    def set_values(self, vals, stream=None):
+        """Replace the nonzero values the kernels use (sr_set_values): fp32 CUDA tensor of
+        out_nnz values in the order sddmm() writes."""
+        import torch
+        if vals.dtype != torch.float32 or not vals.is_cuda or vals.numel() != self.out_nnz or not vals.is_contiguous():
+            raise ValueError("vals must be a contiguous fp32 CUDA tensor of out_nnz values")
+        _check(lib().sr_set_values(self._h, _ptr(vals), _stream(stream)))
+
     def sddmm(self, X, Y, out=None, stream=None):
         """out[p] := vals[p]·<X[row(p)], Y[col(p)]> (Alg 2) in the caller's nnz order."""
         import torch
@@ -284,6 +316,33 @@ class SparseMatrix:
         _check(lib().sr_sddmm(self._h, _ptr(X), X.stride(0), _ptr(Y), Y.stride(0), K, _ptr(out),
                               _stream(stream)))
         return out
+
+
+def trial(cands, op: str, U, V=None, out=None, reps: int = 5, stream=None):
+    """Trial-and-error plan selection (sr_trial, P:267-269): time `op` ("spmm": U = B, out = C;
+    "sddmm": U = X, V = Y) on every candidate SparseMatrix (plans of one matrix, e.g. a
+    reordered one and one in the original order) and return (index of the fastest, [median ms])."""
+    import torch
+    n = len(cands)
+    hs = (C.c_void_p * n)(*[c._h for c in cands])
+    K = U.shape[1]
+    if op == "spmm":
+        code, pv, ldv = SR_OP_SPMM, None, 0
+        if out is None:
+            out = torch.empty((cands[0].out_rows, K), dtype=torch.float32, device=U.device)
+        ldo = out.stride(0)
+    elif op == "sddmm":
+        code, pv, ldv = SR_OP_SDDMM, _ptr(V), V.stride(0)
+        if out is None:
+            out = torch.empty(cands[0].out_nnz, dtype=torch.float32, device=U.device)
+        ldo = 1
+    else:
+        raise ValueError("op must be 'spmm' or 'sddmm'")
+    best = C.c_int32()
+    ms = (C.c_float * n)()
+    _check(lib().sr_trial(C.cast(hs, C.c_void_p), n, code, _ptr(U), U.stride(0), pv, ldv, K, _ptr(out), ldo, reps,
+                          _stream(stream), C.byref(best), C.cast(ms, C.c_void_p)))
+    return best.value, [float(x) for x in ms]
 
 
 # ---------------------------------------------------------------- host-only entry points

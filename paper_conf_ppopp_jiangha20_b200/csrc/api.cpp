@@ -481,6 +481,33 @@ int reorder_round(const int64_t* rowptr, const int32_t* col, int64_t M, const sr
   return SR_OK;
 }
 
+// Shard selection + device execution plan of the plan held in h (perm1, its tiling, perm2).
+int finish_plan(sr_csr_s* h, cudaStream_t s) {
+  const sr_reorder_params* p = &h->params;
+  const Tiling& T = h->tiles;
+  const int64_t M = h->A.M;
+  sr_plan_stats& st = h->stats;
+  // shard: contiguous nnz-balanced panel ranges
+  int64_t pb = 0, pe = T.npanels;
+  if (p->world > 1) {
+    std::vector<int64_t> w((size_t)T.npanels), cuts((size_t)p->world + 1);
+    for (int64_t q = 0; q < T.npanels; ++q) {
+      const int64_t a = q * p->panel_rows, b = std::min<int64_t>(M, a + p->panel_rows);
+      w[q] = (T.drow_ptr[b] - T.drow_ptr[a]) + (T.rrow_ptr[b] - T.rrow_ptr[a]);
+    }
+    partition_panels(T.npanels, w.data(), p->world, cuts.data());
+    pb = cuts[p->rank];
+    pe = cuts[p->rank + 1];
+  }
+  st.shard_panel_begin = pb;
+  st.shard_panel_end = pe;
+  SR_TRY(build_exec_plan(h, pb, pe, s));
+  st.shard_nrows = (int64_t)h->shard_rows.size();
+  st.shard_nnz = (int64_t)h->shard_nnz_ids.size();
+  h->reordered = true;
+  return SR_OK;
+}
+
 }  // namespace
 }  // namespace sr
 
@@ -665,24 +692,7 @@ int sr_reorder(sr_csr h, const sr_reorder_params* p, sr_stream stream) {
   for (int32_t q : order)
     if (T.rrow_ptr[q + 1] > T.rrow_ptr[q]) h->perm2.push_back(q);
   st.n_perm2 = (int64_t)h->perm2.size();
-  // shard: contiguous nnz-balanced panel ranges
-  int64_t pb = 0, pe = T.npanels;
-  if (p->world > 1) {
-    std::vector<int64_t> w((size_t)T.npanels), cuts((size_t)p->world + 1);
-    for (int64_t q = 0; q < T.npanels; ++q) {
-      const int64_t a = q * p->panel_rows, b = std::min<int64_t>(M, a + p->panel_rows);
-      w[q] = (T.drow_ptr[b] - T.drow_ptr[a]) + (T.rrow_ptr[b] - T.rrow_ptr[a]);
-    }
-    partition_panels(T.npanels, w.data(), p->world, cuts.data());
-    pb = cuts[p->rank];
-    pe = cuts[p->rank + 1];
-  }
-  st.shard_panel_begin = pb;
-  st.shard_panel_end = pe;
-  SR_TRY(build_exec_plan(h, pb, pe, s));
-  st.shard_nrows = (int64_t)h->shard_rows.size();
-  st.shard_nnz = (int64_t)h->shard_nnz_ids.size();
-  h->reordered = true;
+  SR_TRY(finish_plan(h, s));
   st.t_total_s = now_s() - t_start;
   return SR_OK;
 }
@@ -852,3 +862,247 @@ int sr_host_partition(int64_t npanels, const int64_t* weights, int32_t G, int64_
 }
 
 }  // extern "C"
+
+// ------------------------------------------------------------------ offline plans
+namespace sr {
+namespace {
+constexpr char kPlanMagic[8] = {'S', 'R', 'P', 'L', 'A', 'N', '0', '1'};
+constexpr uint32_t kPlanVersion = 1;
+
+// 64-bit hash of a byte range (word-wise multiply-xorshift; not cryptographic).
+uint64_t hash_bytes(const void* p, size_t n, uint64_t h) {
+  const unsigned char* b = static_cast<const unsigned char*>(p);
+  size_t i = 0;
+  for (; i + 8 <= n; i += 8) {
+    uint64_t w;
+    std::memcpy(&w, b + i, 8);
+    h ^= w * 0x9E3779B97F4A7C15ull;
+    h = (h << 27 | h >> 37) * 0xBF58476D1CE4E5B9ull;
+  }
+  for (; i < n; ++i) h = (h ^ b[i]) * 0x100000001B3ull;
+  return h ^ (h >> 31);
+}
+
+uint64_t matrix_fingerprint(const HostCSR& A) {
+  uint64_t h = hash_bytes(&A.M, 8, 0x5252504C414E3031ull);
+  h = hash_bytes(&A.N, 8, h);
+  h = hash_bytes(A.rowptr.data(), A.rowptr.size() * 8, h);
+  return hash_bytes(A.col.data(), A.col.size() * 4, h);
+}
+
+struct PlanWriter {
+  std::vector<unsigned char> b;
+  template <typename T>
+  void put(const T& v) { put_raw(&v, sizeof(T)); }
+  void put_raw(const void* p, size_t n) {
+    const unsigned char* c = static_cast<const unsigned char*>(p);
+    b.insert(b.end(), c, c + n);
+  }
+};
+
+struct PlanReader {
+  const unsigned char* p;
+  size_t n, off = 0;
+  bool ok = true;
+  bool get_raw(void* dst, size_t k) {
+    if (!ok || off + k > n) return ok = false;
+    std::memcpy(dst, p + off, k);
+    off += k;
+    return true;
+  }
+  template <typename T>
+  bool get(T& v) { return get_raw(&v, sizeof(T)); }
+};
+}  // namespace
+}  // namespace sr
+
+extern "C" {
+
+int sr_plan_save(sr_csr h, void* buf, int64_t cap, int64_t* len) {
+  if (!h || !len) return einval("sr_plan_save: NULL argument");
+  if (!h->reordered) {
+    set_error("sr_plan_save: the handle has no plan (call sr_reorder or sr_plan_load first)");
+    return SR_ESTATE;
+  }
+  PlanWriter w;
+  w.put_raw(kPlanMagic, 8);
+  w.put(kPlanVersion);
+  w.put((uint32_t)0);
+  w.put(h->A.M);
+  w.put(h->A.N);
+  const int64_t nnz = h->A.nnz();
+  w.put(nnz);
+  w.put(matrix_fingerprint(h->A));
+  sr_reorder_params p = h->params;
+  p.world = 1;
+  p.rank = 0;
+  w.put(p);
+  sr_plan_stats st = h->stats;  // shard fields describe the whole matrix in the image
+  st.shard_panel_begin = 0;
+  st.shard_panel_end = st.npanels;
+  st.shard_nrows = h->A.M;
+  st.shard_nnz = nnz;
+  w.put(st);
+  w.put((int64_t)h->perm1.size());
+  w.put_raw(h->perm1.data(), h->perm1.size() * 4);
+  w.put((int64_t)h->perm2.size());
+  w.put_raw(h->perm2.data(), h->perm2.size() * 4);
+  w.put(hash_bytes(w.b.data(), w.b.size(), 0));
+  *len = (int64_t)w.b.size();
+  if (!buf) return SR_OK;
+  if (cap < *len) return einval("sr_plan_save: capacity too small");
+  std::memcpy(buf, w.b.data(), w.b.size());
+  return SR_OK;
+}
+
+int sr_plan_load(sr_csr h, const void* buf, int64_t len, int32_t world, int32_t rank, sr_stream stream) {
+  if (!h || !buf || len <= 0) return einval("sr_plan_load: NULL argument");
+  if (h->reordered) {
+    set_error("sr_plan_load: the handle already has a plan");
+    return SR_ESTATE;
+  }
+  const double t_start = now_s();
+  PlanReader r{static_cast<const unsigned char*>(buf), (size_t)len};
+  if (len < 8 + 8 || std::memcmp(buf, kPlanMagic, 8) != 0) return einval("sr_plan_load: not a plan image");
+  uint64_t sum = 0;
+  std::memcpy(&sum, r.p + len - 8, 8);
+  if (hash_bytes(buf, (size_t)len - 8, 0) != sum) return einval("sr_plan_load: checksum mismatch (corrupted image)");
+  char magic[8];
+  uint32_t ver = 0, res = 0;
+  int64_t M = 0, N = 0, nnz = 0, len1 = 0, len2 = 0;
+  uint64_t fp = 0;
+  sr_reorder_params p;
+  sr_plan_stats st;
+  r.get_raw(magic, 8);
+  r.get(ver);
+  r.get(res);
+  r.get(M);
+  r.get(N);
+  r.get(nnz);
+  r.get(fp);
+  r.get(p);
+  r.get(st);
+  if (!r.ok || ver != kPlanVersion) return einval("sr_plan_load: unsupported image version");
+  const HostCSR& A = h->A;
+  if (M != A.M || N != A.N || nnz != A.nnz() || fp != matrix_fingerprint(A))
+    return einval("sr_plan_load: the image belongs to another matrix");
+  p.world = world;
+  p.rank = rank;
+  SR_TRY(check_params(&p));
+  if (!r.get(len1) || len1 != M) return einval("sr_plan_load: bad perm1 length");
+  std::vector<int32_t> perm1((size_t)M), perm2;
+  if (!r.get_raw(perm1.data(), (size_t)M * 4) || !r.get(len2) || len2 < 0 || len2 > M)
+    return einval("sr_plan_load: truncated image");
+  perm2.resize((size_t)len2);
+  if (!r.get_raw(perm2.data(), (size_t)len2 * 4) || r.off + 8 != (size_t)len)
+    return einval("sr_plan_load: truncated image");
+  {  // perm1 must be a permutation of [0, M)
+    std::vector<uint8_t> seen((size_t)M, 0);
+    for (int32_t v : perm1) {
+      if (v < 0 || v >= M || seen[v]) return einval("sr_plan_load: perm1 is not a permutation");
+      seen[v] = 1;
+    }
+  }
+  DeviceGuard dg(h->device);
+  cudaStream_t s = stream ? (cudaStream_t)stream : h->init_stream;
+  h->params = p;
+  const double t0 = now_s();
+  Tiling T;
+  tile_rows(A, perm1, p.panel_rows, p.dense_min, T);
+  {  // perm2 must list every non-empty remainder position exactly once
+    std::vector<uint8_t> seen((size_t)M, 0);
+    int64_t nonempty = 0;
+    for (int64_t q = 0; q < M; ++q) nonempty += T.rrow_ptr[q + 1] > T.rrow_ptr[q];
+    for (int32_t q : perm2) {
+      if (q < 0 || q >= M || seen[q] || T.rrow_ptr[q + 1] == T.rrow_ptr[q]) {
+        sr_default_params(&h->params);
+        return einval("sr_plan_load: perm2 does not match the tiling of perm1");
+      }
+      seen[q] = 1;
+    }
+    if (nonempty != len2) {
+      sr_default_params(&h->params);
+      return einval("sr_plan_load: perm2 does not match the tiling of perm1");
+    }
+  }
+  h->perm1 = std::move(perm1);
+  h->perm2 = std::move(perm2);
+  h->tiles = std::move(T);
+  st.t_lsh1_s = st.t_cluster1_s = st.t_lsh2_s = st.t_cluster2_s = 0.0;
+  st.t_tile_s = now_s() - t0;
+  h->stats = st;
+  SR_TRY(finish_plan(h, s));
+  h->stats.t_total_s = now_s() - t_start;
+  return SR_OK;
+}
+
+int sr_trial(const sr_csr* cands, int32_t n, int32_t op, const float* U, int64_t ldu, const float* V, int64_t ldv,
+             int64_t K, float* out, int64_t ldo, int32_t reps, sr_stream stream, int32_t* best, float* ms) {
+  if (!cands || n < 1 || !best || reps < 1) return einval("sr_trial: bad argument");
+  if (op != SR_OP_SPMM && op != SR_OP_SDDMM) return einval("sr_trial: op must be SR_OP_SPMM or SR_OP_SDDMM");
+  for (int32_t i = 0; i < n; ++i) {
+    if (!cands[i]) return einval("sr_trial: NULL candidate");
+    const sr_csr_s* a = cands[0];
+    const sr_csr_s* b = cands[i];
+    const bool sa = a->reordered && a->params.world > 1, sb = b->reordered && b->params.world > 1;
+    if (a->A.M != b->A.M || a->A.N != b->A.N || a->A.nnz() != b->A.nnz() || sa || sb || a->device != b->device)
+      return einval("sr_trial: candidates must be single-GPU plans of one matrix on one device");
+  }
+  DeviceGuard dg(cands[0]->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  cudaEvent_t e0, e1;
+  SR_CUDA_TRY(cudaEventCreate(&e0));
+  if (cudaEventCreate(&e1) != cudaSuccess) {
+    cudaEventDestroy(e0);
+    cudaGetLastError();
+    set_error("sr_trial: cudaEventCreate failed");
+    return SR_ECUDA;
+  }
+  int rc = SR_OK;
+  float best_ms = 0.f;
+  *best = 0;
+  for (int32_t i = 0; i < n && rc == SR_OK; ++i) {
+    auto call = [&]() {
+      return op == SR_OP_SPMM ? sr_spmm(cands[i], U, K, ldu, out, ldo, stream)
+                              : sr_sddmm(cands[i], U, ldu, V, ldv, K, out, stream);
+    };
+    if ((rc = call()) != SR_OK) break;  // warm-up
+    std::vector<float> t((size_t)reps);
+    for (int32_t k = 0; k < reps && rc == SR_OK; ++k) {
+      cudaEventRecord(e0, s);
+      if ((rc = call()) != SR_OK) break;
+      cudaEventRecord(e1, s);
+      if (cudaEventSynchronize(e1) != cudaSuccess || cudaEventElapsedTime(&t[k], e0, e1) != cudaSuccess) {
+        cudaGetLastError();
+        set_error("sr_trial: timing failed");
+        rc = SR_ECUDA;
+      }
+    }
+    if (rc != SR_OK) break;
+    std::sort(t.begin(), t.end());
+    const float med = t[(size_t)reps / 2];
+    if (ms) ms[i] = med;
+    if (i == 0 || med < best_ms) {
+      best_ms = med;
+      *best = i;
+    }
+  }
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  return rc;
+}
+
+}  // extern "C"
+
+extern "C" int sr_set_values(sr_csr h, const float* vals, sr_stream stream) {
+  if (!h) return einval("sr_set_values: NULL handle");
+  const int64_t n = h->reordered ? (int64_t)h->shard_nnz_ids.size() : h->A.nnz();
+  if (n == 0) return SR_OK;
+  if (!vals) return einval("sr_set_values: NULL values");
+  DeviceGuard dg(h->device);
+  DevPlan& P = h->plan;
+  cudaStream_t s = (cudaStream_t)stream;
+  SR_TRY(launch_set_values(P.s_ent.p, P.s_oidx.p, (int64_t)P.s_ent.n, vals, s));
+  if (P.n_units > 0) SR_TRY(launch_set_values(P.d_ent.p, P.d_oidx.p, (int64_t)P.d_ent.n, vals, s));
+  return SR_OK;
+}

@@ -1661,7 +1661,25 @@ __global__ void scatter_values_kernel(const float* __restrict__ src, const int64
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n && ids[i] >= 0) dst[ids[i]] = src[i];
 }
+
+// sr_set_values: ent[e].y := vals[oidx[e]] (oidx = the SDDMM output index of each plan entry,
+// i.e. the handle's output order; padding entries carry -1)
+__global__ void set_values_kernel(int2* __restrict__ ent, const int32_t* __restrict__ oidx, int64_t n,
+                                  const float* __restrict__ vals) {
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t o = __ldg(oidx + e);
+    if (o >= 0) ent[e].y = __float_as_int(__ldg(vals + o));
+  }
+}
 }  // namespace
+
+int launch_set_values(int2* ent, const int32_t* oidx, int64_t n, const float* vals, cudaStream_t s) {
+  if (n == 0) return SR_OK;
+  const unsigned grid = (unsigned)std::min<int64_t>((n + 255) / 256, (int64_t)num_sms() * 8);
+  set_values_kernel<<<grid, 256, 0, s>>>(ent, oidx, n, vals);
+  SR_CUDA_TRY(cudaGetLastError());
+  return SR_OK;
+}
 
 int launch_scatter_rows(const float* src, int64_t lds, const int32_t* rows, int64_t n, int64_t K, float* dst,
                         int64_t ldd, cudaStream_t s) {

@@ -59,8 +59,9 @@ struct DevBuf {
     n = count;
     return SR_OK;
   }
-  int upload(const T* host, size_t count, cudaStream_t s) {
+  int upload(const T* host, size_t count, cudaStream_t s) {  // n = count (0 allowed)
     SR_TRY(alloc(count));
+    n = count;
     if (count) SR_CUDA_TRY(cudaMemcpyAsync(p, host, count * sizeof(T), cudaMemcpyHostToDevice, s));
     return SR_OK;
   }
@@ -219,4 +220,5 @@ int launch_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64
 int launch_scatter_rows(const float* src, int64_t lds, const int32_t* rows, int64_t n, int64_t K, float* dst,
                         int64_t ldd, cudaStream_t s);
 int launch_scatter_values(const float* src, const int64_t* ids, int64_t n, float* dst, cudaStream_t s);
+int launch_set_values(int2* ent, const int32_t* oidx, int64_t n, const float* vals, cudaStream_t s);
 }  // namespace sr

@@ -98,3 +98,21 @@ def test_host_partition_matches_oracle(sr, oracle, G):
         w = rng.integers(0, 1000, size=int(rng.integers(1, 300)))
         w[rng.random(w.size) < 0.2] = 0
         np.testing.assert_array_equal(sr.host_partition(w, G), oracle.partition(w, G))
+
+
+def test_transpose_csr_matches_dense():
+    """cf.transpose_csr (host helper of the CF loop): Aᵀ and the nnz permutation."""
+    import numpy as np
+    from paper_conf_ppopp_jiangha20_b200.cf import transpose_csr
+    from synth import generators as g
+    A = g.random_csr(40, 30, 0.2, 3, empty_frac=0.1)
+    trp, tcol, perm = transpose_csr(A.nrows, A.ncols, A.rowptr, A.colidx)
+    D = np.zeros((A.nrows, A.ncols))
+    rows = np.repeat(np.arange(A.nrows), np.diff(A.rowptr))
+    D[rows, A.colidx] = A.vals
+    T = np.zeros((A.ncols, A.nrows))
+    trows = np.repeat(np.arange(A.ncols), np.diff(trp))
+    T[trows, tcol] = A.vals[perm]
+    np.testing.assert_array_equal(T, D.T)
+    for r in range(A.ncols):  # columns sorted within each row of Aᵀ
+        assert np.all(np.diff(tcol[trp[r]:trp[r + 1]]) > 0)
