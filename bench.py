@@ -50,9 +50,10 @@ def parse():
     ap.add_argument("--tile-cols", type=int, default=64)
     ap.add_argument("--max-bucket", type=int, default=32)
     # ASpT dense-column threshold (R17).  The paper's example is 2 (a P100 with 64 KB of
-    # shared memory per SM); on B200 (126 MB L2, 128-bit gathers at 8 CTAs/SM) staging pays only
-    # for columns shared by about half the panel: sweep in profiles/r01/NOTES.md.
-    ap.add_argument("--dense-min", type=int, default=32)
+    # shared memory per SM); on B200 (126 MB L2, row-group task kernels gathering from L2 at ~15 TB/s)
+    # staging pays only for columns shared by (nearly) the whole 64-row panel: sweeps in
+    # profiles/r01/NOTES.md (session 3: 64 best with tiles present, equal to no tiles).
+    ap.add_argument("--dense-min", type=int, default=64)
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target CPU work of cpu_baseline")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -221,33 +222,25 @@ def gathered_bytes(kind: str, tm: dict, K: int) -> float:
     return row * (tm["sparse_nnz"] if kind.endswith("sparse_rows") else tm["dense_col_loads"])
 
 
-def gather_ceiling(table_bytes: float, K: int):
-    """Measured random-row-gather bandwidth for a table of this size (profiles/gather_bw.cu,
-    committed results in profiles/r01/gather_bw.jsonl; 8 CTAs/SM series), log-interpolated in
-    the table size, nearest row width (128 or 512 bytes)."""
+def gather_ceiling(K: int):
+    """Measured ceiling of random row gathers that HIT the L2 (profiles/gather_bw.cu, committed
+    results in profiles/r01/gather_bw.jsonl: the largest rate over the L2-resident table sizes
+    <= 64 MB, 8 CTAs/SM, nearest row width 128 or 512 bytes).  Every gathered row of phase S
+    crosses the L2 -> SM path once, so gathered bytes / this rate bounds the kernel's time from
+    below whatever its L2 hit rate (misses only add HBM time)."""
     path = os.path.join(ROOT, "profiles", "r01", "gather_bw.jsonl")
     if not os.path.exists(path):
         return None, None
-    pts = []
     rb = 512 if K * 4 >= 320 else 128
+    best = None
     with open(path) as f:
         for line in f:
             d = json.loads(line)
-            if d.get("row_bytes") == rb and d.get("ctas_per_sm") == 8:
-                pts.append((d["table_MB"] * 2.0 ** 20, d["gather_GBs"]))
-    if not pts:
+            if d.get("row_bytes") == rb and d.get("ctas_per_sm") == 8 and d.get("table_MB", 1e9) <= 64:
+                best = max(best or 0.0, d["gather_GBs"])
+    if best is None:
         return None, None
-    pts.sort()
-    import math
-    x = min(max(table_bytes, pts[0][0]), pts[-1][0])
-    for (x0, y0), (x1, y1) in zip(pts, pts[1:]):
-        if x0 <= x <= x1:
-            w = (math.log(x) - math.log(x0)) / (math.log(x1) - math.log(x0)) if x1 > x0 else 0.0
-            y = y0 + w * (y1 - y0)
-            break
-    else:
-        y = pts[-1][1]
-    return y, f"profiles/r01/gather_bw.jsonl: random {rb}-byte row gathers, {table_bytes / 2**20:.0f} MB table (interpolated)"
+    return best, f"profiles/r01/gather_bw.jsonl: L2-resident random {rb}-byte row gathers (max over <= 64 MB tables)"
 
 
 def run_ours(args, A, ops, rank, world, local_rank):
@@ -351,16 +344,17 @@ def run_ours(args, A, ops, rank, world, local_rank):
                     "frac": d["achieved_gbs"] / peak, "traffic": traffic, "peak_source": peak_src,
                     "algorithmic_bytes_per_launch": d["algorithmic_bytes"], "avg_ms": d["avg_ms"]}
 
-    # the same kernel against the measured random-gather ceiling of its operand's size: the
-    # gathered rows come from L2/HBM at a rate set by the table size (profiles/r01/NOTES.md)
+    # the same kernel against the L2 -> SM gather ceiling (the path every gathered row takes;
+    # DESIGN.md §5): a conservative efficiency for a gather-bound kernel whose HBM bytes are
+    # far below the bytes it moves into the SMs
     gather_roof = None
     if dom:
         d = kern[dom]
         gb = gathered_bytes(dom, tm, K)
-        ceil_gbs, ceil_src = gather_ceiling(4.0 * K * A.ncols, K)
+        ceil_gbs, ceil_src = gather_ceiling(K)
         if ceil_gbs:
             ach = gb / (d["avg_ms"] / 1e3) / 1e9
-            gather_roof = {"kernel": dom, "bound": "gather", "achieved": ach, "peak": ceil_gbs, "unit": "GB/s",
+            gather_roof = {"kernel": dom, "bound": "l2_gather", "achieved": ach, "peak": ceil_gbs, "unit": "GB/s",
                            "frac": ach / ceil_gbs, "gathered_bytes_per_launch": gb, "peak_source": ceil_src}
 
     # end to end through the public API with host buffers (pinned), per step

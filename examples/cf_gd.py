@@ -7,7 +7,7 @@ line: preprocessing seconds, device ms per iteration (CUDA events, median), the 
 preprocessing to one iteration (the paper's Tables 3/4 quantity), the iterations after which
 reordering has paid for itself against the original-order plans, and the loss trajectory.
 
-  python examples/cf_gd.py [--config cf] [--K 128] [--iters 20] [--lr 1e-4]
+  python examples/cf_gd.py [--config cf] [--K 128] [--iters 20] [--lr 1e-6]
 """
 from __future__ import annotations
 
@@ -48,8 +48,8 @@ def main():
     ap.add_argument("--config", default="cf", choices=list(gen.CONFIGS))
     ap.add_argument("--K", type=int, default=128)
     ap.add_argument("--iters", type=int, default=20)
-    ap.add_argument("--lr", type=float, default=1e-4)
-    ap.add_argument("--dense-min", type=int, default=32)
+    ap.add_argument("--lr", type=float, default=1e-6)
+    ap.add_argument("--dense-min", type=int, default=64)
     args = ap.parse_args()
     import paper_conf_ppopp_jiangha20_b200 as sr
     R = gen.make(args.config)

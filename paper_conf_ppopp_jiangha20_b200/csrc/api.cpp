@@ -153,6 +153,10 @@ int upload_items(DevPlan& P, ItemBuilder& ib, int64_t n_sddmm_items, cudaStream_
   const std::vector<int4> tasks = build_tasks(ib, (int64_t)ib.items.size(), 32);
   P.n_tasks = (int64_t)tasks.size();
   SR_TRY(P.tasks.upload(tasks, s));
+  // narrow-K SpMM: one task per lane group, at most 8 rows (one per lane of an 8-lane group)
+  const std::vector<int4> tasks8 = build_tasks(ib, (int64_t)ib.items.size(), 8);
+  P.n_tasks8 = (int64_t)tasks8.size();
+  SR_TRY(P.tasks8.upload(tasks8, s));
   // SDDMM: the non-empty items only (a prefix), at most 8 rows per task (X rows staged in smem)
   const std::vector<int4> stasks = build_tasks(ib, n_sddmm_items, 8);
   P.n_stasks = (int64_t)stasks.size();
@@ -942,6 +946,7 @@ int sr_plan_save(sr_csr h, void* buf, int64_t cap, int64_t* len) {
   st.shard_panel_end = st.npanels;
   st.shard_nrows = h->A.M;
   st.shard_nnz = nnz;
+  st.t_lsh1_s = st.t_cluster1_s = st.t_tile_s = st.t_lsh2_s = st.t_cluster2_s = st.t_total_s = 0.0;  // canonical
   w.put(st);
   w.put((int64_t)h->perm1.size());
   w.put_raw(h->perm1.data(), h->perm1.size() * 4);

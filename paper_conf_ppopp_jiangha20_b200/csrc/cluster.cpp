@@ -10,6 +10,10 @@
 //  * candidate-pair membership (line 27, R9) is an open-addressing hash set.
 // Readings R3-R12 decide everything the paper leaves open.
 #include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
+#include <parallel/algorithm>
 #include <cstring>
 #include <numeric>
 #include <queue>
@@ -54,6 +58,16 @@ class PairSet {
       h = (h + 1) & mask_;
     }
   }
+  // concurrent insert of keys known to be distinct (initial build, OpenMP): CAS on the slot
+  void insert_distinct_concurrent(uint64_t k) {
+    size_t h = hash(k) & mask_;
+    while (true) {
+      uint64_t expected = kEmpty;
+      if (__atomic_compare_exchange_n(&slots_[h], &expected, k, false, __ATOMIC_RELAXED, __ATOMIC_RELAXED)) return;
+      h = (h + 1) & mask_;
+    }
+  }
+  void set_size(size_t n) { size_ = n; }
   void insert(uint64_t k) {
     if (2 * (size_ + 1) > slots_.size()) grow();
     size_t h = hash(k) & mask_;
@@ -92,8 +106,21 @@ inline void intersect(const int64_t* rowptr, const int32_t* col, int64_t a, int6
                       uint32_t* inter, uint32_t* uni) {
   const int32_t *p = col + rowptr[a], *pe = col + rowptr[a + 1];
   const int32_t *q = col + rowptr[b], *qe = col + rowptr[b + 1];
-  const int64_t na = pe - p, nb = qe - q;
+  int64_t na = pe - p, nb = qe - q;
   int64_t n = 0;
+  if (na > nb) {
+    std::swap(p, q);
+    std::swap(pe, qe);
+  }
+  if ((qe - q) >= 16 * (pe - p)) {  // skewed sizes (hub rows): binary-search the short list's
+    for (; p < pe && q < qe; ++p) {  // columns in the long one, O(short · log long)
+      q = std::lower_bound(q, qe, *p);
+      if (q < qe && *q == *p) ++n, ++q;
+    }
+    *inter = (uint32_t)n;
+    *uni = (uint32_t)(na + nb - n);
+    return;
+  }
   while (p < pe && q < qe) {
     const int32_t x = *p, y = *q;
     n += (x == y);
@@ -109,9 +136,14 @@ inline void intersect(const int64_t* rowptr, const int32_t* col, int64_t a, int6
 void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t npairs,
                   const uint64_t* pairs, const uint32_t* inter, const uint32_t* uni,
                   int32_t threshold_size, int32_t* perm) {
-  // initial candidates in heap order
+  const bool dbg = getenv("SR_DEBUG_CLUSTER") != nullptr;
+  auto now = [] { return std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count(); };
+  double t0 = now();
+  // initial candidates in heap order; the membership set is built in parallel (the pairs are
+  // distinct), the heap order is a strict total order (R10) so any sort gives the same array
   std::vector<Cand> init((size_t)npairs);
   PairSet members((size_t)npairs + (size_t)npairs / 4);
+#pragma omp parallel for schedule(static)
   for (int64_t e = 0; e < npairs; ++e) {
     Cand c;
     c.i = (uint32_t)(pairs[e] >> 32);
@@ -124,11 +156,15 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
     }
     if (c.uni == 0) c.uni = 1;  // J(empty, empty) := 0/1 (R16)
     init[e] = c;
-    members.insert(pairs[e]);
+    members.insert_distinct_concurrent(pairs[e]);
   }
+  members.set_size((size_t)npairs);
   bool sorted = true;
   for (int64_t e = 1; e < npairs && sorted; ++e) sorted = !before(init[e], init[e - 1]);
-  if (!sorted) std::stable_sort(init.begin(), init.end(), before);
+  const double t1 = now();
+  if (!sorted) __gnu_parallel::sort(init.begin(), init.end(), before);
+  const double t2 = now();
+  int64_t n_reinsert = 0, n_pops = 0;
 
   std::vector<int32_t> cid((size_t)M), csz((size_t)M, 1);
   std::vector<uint8_t> dead((size_t)M, 0);
@@ -178,8 +214,13 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
       if (c.uni == 0) c.uni = 1;
       extra.push(c);
       members.insert(key);
+      ++n_reinsert;
     }
   }
+  if (dbg)
+    fprintf(stderr, "cluster_rows: build %.3f s, sort %.3f s (sorted=%d), loop %.3f s, %lld re-inserted\n", t1 - t0,
+            t2 - t1, (int)sorted, now() - t2, (long long)n_reinsert);
+  (void)n_pops;
   // rule B (R11): clusters of >= 2 rows by ascending root, then singletons ascending
   std::vector<int32_t> r_of((size_t)M);
   std::vector<int64_t> count((size_t)M + 1, 0);

@@ -281,11 +281,11 @@ def test_full_size_sampled(env, oracle, config):
     plus the 20 longest rows (K=128, and K=32 for C2); SDDMM on every nnz of those rows."""
     sr, torch = env
     A = g.make(config)
-    # C2 (rmat) is bench.py's workload: its plan (dense_min 32, profiles/r01/NOTES.md); the other
+    # C2 (rmat) is bench.py's workload: its plan (dense_min 64, profiles/r01/NOTES.md); the other
     # configs keep the paper's example threshold 2 (P:111), under which AUTO skips their round 1
     # (DenseRatio0 > 1/10) and the CPU oracle's plan finishes in minutes
     kw = dict(siglen=128, bsize=2, seed=4, max_bucket=32, threshold_size=256, panel_rows=64,
-              dense_min=32 if config == "rmat" else 2, mode=0)
+              dense_min=64 if config == "rmat" else 2, mode=0)
     M = sr.SparseMatrix.from_csr(A)
     M.reorder(sr.default_params(**kw))
     ref = oracle.plan(A, **kw)
