@@ -343,6 +343,19 @@ def run_ours(args, A, ops, rank, world, local_rank):
         roofline = {"kernel": dom, "bound": "hbm", "achieved": d["achieved_gbs"], "peak": peak, "unit": "GB/s",
                     "frac": d["achieved_gbs"] / peak, "traffic": traffic, "peak_source": peak_src,
                     "algorithmic_bytes_per_launch": d["algorithmic_bytes"], "avg_ms": d["avg_ms"]}
+        if traffic:
+            # north_star's "achieved HBM GB/s": ncu DRAM bytes per launch / this run's launch time
+            roofline["dram_gbs"] = traffic / (d["avg_ms"] / 1e3) / 1e9
+            roofline["dram_frac"] = roofline["dram_gbs"] / peak
+        # the same for every kernel with an ncu record
+        if os.path.exists(prof_path) and world == 1:
+            with open(prof_path) as f:
+                tr_all = json.load(f)
+            for k, dk in kern.items():
+                rec = tr_all.get(f"{args.config}_K{K}_{k}")
+                if rec is not None:
+                    dk["dram_bytes_ncu"] = rec["bytes"]
+                    dk["dram_gbs"] = rec["bytes"] / (dk["avg_ms"] / 1e3) / 1e9
 
     # the same kernel against the L2 -> SM gather ceiling (the path every gathered row takes;
     # DESIGN.md §5): a conservative efficiency for a gather-bound kernel whose HBM bytes are

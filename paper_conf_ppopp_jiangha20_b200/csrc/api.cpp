@@ -153,10 +153,6 @@ int upload_items(DevPlan& P, ItemBuilder& ib, int64_t n_sddmm_items, cudaStream_
   const std::vector<int4> tasks = build_tasks(ib, (int64_t)ib.items.size(), 32);
   P.n_tasks = (int64_t)tasks.size();
   SR_TRY(P.tasks.upload(tasks, s));
-  // narrow-K SpMM: one task per lane group, at most 8 rows (one per lane of an 8-lane group)
-  const std::vector<int4> tasks8 = build_tasks(ib, (int64_t)ib.items.size(), 8);
-  P.n_tasks8 = (int64_t)tasks8.size();
-  SR_TRY(P.tasks8.upload(tasks8, s));
   // SDDMM: the non-empty items only (a prefix), at most 8 rows per task (X rows staged in smem)
   const std::vector<int4> stasks = build_tasks(ib, n_sddmm_items, 8);
   P.n_stasks = (int64_t)stasks.size();

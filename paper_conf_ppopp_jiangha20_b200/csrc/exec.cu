@@ -324,7 +324,8 @@ __global__ void __launch_bounds__(256, MINB) spmm_task_kernel(
   const int lane = threadIdx.x & 31;
   // warp-uniform values through lane-0 shuffles, so the compiler sees uniform control flow
   // (no divergent-shuffle fallback paths and no stack frame)
-  const int64_t w = (int64_t)blockIdx.x * (blockDim.x >> 5) + __shfl_sync(FULL, threadIdx.x >> 5, 0);
+  const int wid = __shfl_sync(FULL, threadIdx.x >> 5, 0);
+  const int64_t w = (int64_t)blockIdx.x * (blockDim.x >> 5) + wid;
   if (w >= n_tasks) return;
   int4 t = __ldg(tasks + w);  // {e0, e1, first item, end item}
   t.x = __shfl_sync(FULL, t.x, 0); t.y = __shfl_sync(FULL, t.y, 0);
@@ -403,116 +404,6 @@ __global__ void __launch_bounds__(256, MINB) spmm_task_kernel(
             acc = make_float4(0.f, 0.f, 0.f, 0.f);
             ++r;
             row_end = t.x + __shfl_sync(FULL, end, r & 31);
-          }
-        }
-      }
-    }
-  }
-}
-
-// ------------------------------------------------------------------ phase S: SpMM, narrow K
-// K = 4·LPG < 128 (K 32: LPG 8): each LPG-lane group of a warp runs its own task (tasks of at
-// most 8 rows, api.cpp: build_tasks), exactly as spmm_task_kernel does with the whole warp —
-// streaming the task's entries with U gathers of K·4 bytes in flight across row boundaries.
-// Groups diverge freely: every shuffle names only its group's lanes.
-template <int LPG, int U, int MINB>
-__global__ void __launch_bounds__(256, MINB) spmm_gtask_kernel(
-    const int4* __restrict__ tasks, int64_t n_tasks, const Item* __restrict__ items,
-    const uint32_t* __restrict__ meta, const int2* __restrict__ ent, const float* __restrict__ B, uint32_t ldb,
-    float* __restrict__ C, int64_t ldc, int K, float* __restrict__ scratch,
-    const int2* __restrict__ split_info, int* __restrict__ split_counter) {
-  constexpr int G = 32 / LPG;
-  const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
-  const unsigned gm = (LPG == 32 ? FULL : ((1u << LPG) - 1u)) << (g * LPG);
-  const int64_t w = (int64_t)blockIdx.x * (blockDim.x >> 5) + __shfl_sync(FULL, threadIdx.x >> 5, 0);
-  const int64_t tid = w * G + g;
-  if (tid >= n_tasks) return;  // whole groups leave together
-  const int4 t = __ldg(tasks + tid);  // {e0, e1, first item, end item}, same for the group's lanes
-  const float* Bk = B + lg * 4;
-  const uint32_t m0 = __ldg(meta + t.z);
-  if (m0 & kItemSplit) {  // one chunk of a long row -> scratch; the last chunk combines in order
-    float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-    for (int eb = t.x; eb < t.y; eb += LPG) {
-      const int n = min(LPG, t.y - eb);
-      const int2 my = lg < n ? __ldcs(ent + eb + lg) : make_int2(0, 0);
-      for (int base = 0; base < n; base += U) {
-        float4 b[U];
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-          const int c = __shfl_sync(gm, my.x, min(base + u, n - 1), LPG);
-          b[u] = __ldg(reinterpret_cast<const float4*>(reinterpret_cast<const char*>(Bk) + (uint64_t)(uint32_t)c * ldb));
-        }
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-          const float a = __int_as_float(__shfl_sync(gm, my.y, min(base + u, n - 1), LPG));
-          if (base + u < n) {
-            acc.x = fmaf(a, b[u].x, acc.x); acc.y = fmaf(a, b[u].y, acc.y);
-            acc.z = fmaf(a, b[u].z, acc.z); acc.w = fmaf(a, b[u].w, acc.w);
-          }
-        }
-      }
-    }
-    float* sc = scratch + lg * 4;
-    *reinterpret_cast<float4*>(sc + (int64_t)(m0 & kItemSlotMask) * K) = acc;
-    __threadfence();
-    __syncwarp(gm);
-    const int2 si = __ldg(split_info + (m0 & kItemSlotMask));
-    int last = 0;
-    if (lg == 0) last = (atomicAdd(split_counter + si.x, 1) == si.y - 1);
-    last = __shfl_sync(gm, last, 0, LPG);
-    if (!last) return;
-    __threadfence();
-    float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
-    for (int c = 0; c < si.y; ++c) {
-      const float4 p = __ldcg(reinterpret_cast<const float4*>(sc + (int64_t)(si.x + c) * K));
-      s.x += p.x; s.y += p.y; s.z += p.z; s.w += p.w;
-    }
-    const int o = __ldg(reinterpret_cast<const int4*>(items) + t.z).w;
-    task_store(s, (uint32_t)o | ((m0 & kItemRMW) ? 0x80000000u : 0u), C, ldc, lg);
-    if (lg == 0) split_counter[si.x] = 0;
-    return;
-  }
-  const int cnt = t.w - t.z;  // <= 8 <= LPG rows
-  int end = 0;
-  uint32_t o = 0;
-  if (lg < cnt) {
-    const int4 it = __ldg(reinterpret_cast<const int4*>(items) + t.z + lg);
-    end = it.y - it.x;
-    o = (uint32_t)it.w | ((__ldg(meta + t.z + lg) & kItemRMW) ? 0x80000000u : 0u);
-  }
-  if (t.x == t.y) {  // zero rows
-    for (int r = 0; r < cnt; ++r) task_store(make_float4(0.f, 0.f, 0.f, 0.f), __shfl_sync(gm, o, r, LPG), C, ldc, lg);
-    return;
-  }
-#pragma unroll
-  for (int d = 1; d < LPG; d <<= 1) {
-    const int v = __shfl_up_sync(gm, end, d, LPG);
-    if (lg >= d) end += v;
-  }
-  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-  int r = 0;
-  int row_end = t.x + __shfl_sync(gm, end, 0, LPG);
-  for (int eb = t.x; eb < t.y; eb += LPG) {
-    const int n = min(LPG, t.y - eb);
-    const int2 my = lg < n ? __ldcs(ent + eb + lg) : make_int2(0, 0);
-    for (int base = 0; base < n; base += U) {
-      float4 b[U];
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const int c = __shfl_sync(gm, my.x, min(base + u, n - 1), LPG);
-        b[u] = __ldg(reinterpret_cast<const float4*>(reinterpret_cast<const char*>(Bk) + (uint64_t)(uint32_t)c * ldb));
-      }
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const float a = __int_as_float(__shfl_sync(gm, my.y, min(base + u, n - 1), LPG));
-        if (base + u < n) {
-          acc.x = fmaf(a, b[u].x, acc.x); acc.y = fmaf(a, b[u].y, acc.y);
-          acc.z = fmaf(a, b[u].z, acc.z); acc.w = fmaf(a, b[u].w, acc.w);
-          if (eb + base + u + 1 == row_end) {
-            task_store(acc, __shfl_sync(gm, o, r, LPG), C, ldc, lg);
-            acc = make_float4(0.f, 0.f, 0.f, 0.f);
-            ++r;
-            row_end = t.x + __shfl_sync(gm, end, r & (LPG - 1), LPG);
           }
         }
       }
@@ -1576,26 +1467,6 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
         case 5: tk(spmm_task_kernel<8, 4>); break;
         case 6: tk(spmm_task_kernel<2, 8>); break;
         default: tk(spmm_task_kernel<4, 8>); break;
-      }
-      SR_CUDA_TRY(cudaGetLastError());
-      if (P.profiling) SR_TRY(prof_end(P, s));
-      ++*launches;
-      return SR_OK;
-    }
-    if ((LPG == 8 || LPG == 16) && VEC == 4 && K == 4 * LPG && ldb * 4 < (1ll << 32) && var >= 8 && var <= 10 &&
-        P.n_tasks8 > 0) {  // group tasks (experiment: SR_SPARSE_VARIANT 8-10)
-      constexpr int GG = 32 / LPG;
-      const unsigned tgrid = (unsigned)((P.n_tasks8 + kSparseWarps * GG - 1) / (kSparseWarps * GG));
-      auto tk = [&](auto kern) {
-        kern<<<tgrid, kSparseWarps * 32, 0, s>>>(P.tasks8.p, P.n_tasks8, P.items.p, P.item_meta.p, P.s_ent.p, B,
-                                                  (uint32_t)(ldb * 4), C, ldc, (int)K, P.scratch.p, P.split_info.p,
-                                                  P.split_counter.p);
-      };
-      constexpr int LP = (LPG == 8 || LPG == 16) ? LPG : 8;
-      switch (var) {
-        case 9: tk(spmm_gtask_kernel<LP, 2, 8>); break;
-        case 10: tk(spmm_gtask_kernel<LP, 8, 4>); break;
-        default: tk(spmm_gtask_kernel<LP, 4, 8>); break;
       }
       SR_CUDA_TRY(cudaGetLastError());
       if (P.profiling) SR_TRY(prof_end(P, s));

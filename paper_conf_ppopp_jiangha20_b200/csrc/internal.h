@@ -156,8 +156,6 @@ struct DevPlan {
   int64_t n_items = 0;
   DevBuf<int4> tasks;         // SpMM row-group tasks {e0, e1, first item, end item} (build_tasks)
   int64_t n_tasks = 0;
-  DevBuf<int4> tasks8;        // SpMM tasks of <= 8 rows for the narrow-K group kernel
-  int64_t n_tasks8 = 0;
   DevBuf<int4> stasks;        // SDDMM row-group tasks (<= 8 rows each, non-empty rows only)
   int64_t n_stasks = 0;
   DevBuf<Item> sitems;        // SDDMM items (remainder rows / chunks only)
