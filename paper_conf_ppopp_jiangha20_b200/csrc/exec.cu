@@ -278,44 +278,47 @@ __global__ void __launch_bounds__(256, MINB) sddmm_sparse_kernel(
 // once per task and short rows no longer limit the gathers in flight.  Each launch covers 128
 // columns (one float4 per lane; the host offsets B and C for K = 128·passes).  Rows are still
 // summed in CSR order, chunks of split rows combined in chunk order (deterministic).
-template <int U>
-__device__ __forceinline__ float4 task_row_sum(const int2* __restrict__ ent, int e0, int e1, const float* Bk,
-                                               uint32_t ldb, int lane) {
-  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+template <int U, int VEC>
+__device__ __forceinline__ Frag<VEC> task_row_sum(const int2* __restrict__ ent, int e0, int e1, const float* Bk,
+                                                  uint32_t ldb) {
+  const int lane = threadIdx.x & 31;
+  Frag<VEC> acc;
+  acc.zero();
   for (int eb = e0; eb < e1; eb += 32) {
     const int n = min(32, e1 - eb);
     const int2 my = lane < n ? __ldcs(ent + eb + lane) : make_int2(0, 0);
     for (int base = 0; base < n; base += U) {
-      float4 b[U];
+      Frag<VEC> b[U];
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         // past the end: re-load the last entry's row (same lines, no predicate, no zero fill)
         const int c = __shfl_sync(FULL, my.x, min(base + u, n - 1));
-        b[u] = __ldg(reinterpret_cast<const float4*>(reinterpret_cast<const char*>(Bk) + (uint64_t)(uint32_t)c * ldb));
+        b[u].load_g(reinterpret_cast<const float*>(reinterpret_cast<const char*>(Bk) + (uint64_t)(uint32_t)c * ldb));
       }
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         const float a = __int_as_float(__shfl_sync(FULL, my.y, base + u));
-        if (base + u < n) {
-          acc.x = fmaf(a, b[u].x, acc.x); acc.y = fmaf(a, b[u].y, acc.y);
-          acc.z = fmaf(a, b[u].z, acc.z); acc.w = fmaf(a, b[u].w, acc.w);
-        }
+        if (base + u < n) acc.fma(a, b[u]);
       }
     }
   }
   return acc;
 }
 
-__device__ __forceinline__ void task_store(float4 v, uint32_t o, float* __restrict__ C, int64_t ldc, int lane) {
-  float4* dst = reinterpret_cast<float4*>(C + (int64_t)(o & 0x7fffffffu) * ldc) + lane;
+template <int VEC>
+__device__ __forceinline__ void task_store(Frag<VEC> v, uint32_t o, float* __restrict__ C, int64_t ldc) {
+  float* dst = C + (int64_t)(o & 0x7fffffffu) * ldc + (threadIdx.x & 31) * VEC;
   if (o >> 31) {  // the row also has dense-tile entries (phase D ran first): read-modify-write
-    const float4 old = __ldcg(dst);
-    v.x += old.x; v.y += old.y; v.z += old.z; v.w += old.w;
+    Frag<VEC> old;
+    old.load_cg(dst);
+    v.add(old);
   }
-  __stcs(dst, v);
+  v.store_cs(dst);
 }
 
-template <int U, int MINB>
+// VEC 4: a launch covers 128 columns (one float4 per lane); VEC 1: 32 columns (K = 32·passes,
+// one float per lane, 128-byte gathers).  The host offsets B and C per pass; ldb is in bytes.
+template <int U, int MINB, int VEC>
 __global__ void __launch_bounds__(256, MINB) spmm_task_kernel(
     const int4* __restrict__ tasks, int64_t n_tasks, const Item* __restrict__ items,
     const uint32_t* __restrict__ meta, const int2* __restrict__ ent, const float* __restrict__ B, uint32_t ldb,
@@ -324,18 +327,17 @@ __global__ void __launch_bounds__(256, MINB) spmm_task_kernel(
   const int lane = threadIdx.x & 31;
   // warp-uniform values through lane-0 shuffles, so the compiler sees uniform control flow
   // (no divergent-shuffle fallback paths and no stack frame)
-  const int wid = __shfl_sync(FULL, threadIdx.x >> 5, 0);
-  const int64_t w = (int64_t)blockIdx.x * (blockDim.x >> 5) + wid;
+  const int64_t w = (int64_t)blockIdx.x * (blockDim.x >> 5) + __shfl_sync(FULL, threadIdx.x >> 5, 0);
   if (w >= n_tasks) return;
   int4 t = __ldg(tasks + w);  // {e0, e1, first item, end item}
   t.x = __shfl_sync(FULL, t.x, 0); t.y = __shfl_sync(FULL, t.y, 0);
   t.z = __shfl_sync(FULL, t.z, 0); t.w = __shfl_sync(FULL, t.w, 0);
-  const float* Bk = B + lane * 4;   // B, C are offset to this launch's 128 columns; ldb in bytes
+  const float* Bk = B + lane * VEC;
   const uint32_t m0 = __ldg(meta + t.z);
   if (m0 & kItemSplit) {  // one chunk of a long row -> scratch; the last chunk combines in order
-    const float4 acc = task_row_sum<U>(ent, t.x, t.y, Bk, ldb, lane);
-    float* sc = scratch + k0 + lane * 4;
-    *reinterpret_cast<float4*>(sc + (int64_t)(m0 & kItemSlotMask) * K) = acc;
+    const Frag<VEC> acc = task_row_sum<U, VEC>(ent, t.x, t.y, Bk, ldb);
+    float* sc = scratch + k0 + lane * VEC;
+    acc.store(sc + (int64_t)(m0 & kItemSlotMask) * K);
     __threadfence();
     __syncwarp();
     const int2 si = __ldg(split_info + (m0 & kItemSlotMask));
@@ -344,21 +346,23 @@ __global__ void __launch_bounds__(256, MINB) spmm_task_kernel(
     last = __shfl_sync(FULL, last, 0);
     if (!last) return;
     __threadfence();
-    float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
+    Frag<VEC> s;
+    s.zero();
     int c = 0;
     for (; c + 4 <= si.y; c += 4) {
-      float4 p[4];
+      Frag<VEC> p[4];
 #pragma unroll
-      for (int i = 0; i < 4; ++i) p[i] = __ldcg(reinterpret_cast<const float4*>(sc + (int64_t)(si.x + c + i) * K));
+      for (int i = 0; i < 4; ++i) p[i].load_cg(sc + (int64_t)(si.x + c + i) * K);
 #pragma unroll
-      for (int i = 0; i < 4; ++i) { s.x += p[i].x; s.y += p[i].y; s.z += p[i].z; s.w += p[i].w; }
+      for (int i = 0; i < 4; ++i) s.add(p[i]);
     }
     for (; c < si.y; ++c) {
-      const float4 p = __ldcg(reinterpret_cast<const float4*>(sc + (int64_t)(si.x + c) * K));
-      s.x += p.x; s.y += p.y; s.z += p.z; s.w += p.w;
+      Frag<VEC> p;
+      p.load_cg(sc + (int64_t)(si.x + c) * K);
+      s.add(p);
     }
     const int o = __ldg(reinterpret_cast<const int4*>(items) + t.z).w;
-    task_store(s, (uint32_t)o | ((m0 & kItemRMW) ? 0x80000000u : 0u), C, ldc, lane);
+    task_store<VEC>(s, (uint32_t)o | ((m0 & kItemRMW) ? 0x80000000u : 0u), C, ldc);
     if (lane == 0) split_counter[si.x] = 0;
     return;
   }
@@ -371,7 +375,9 @@ __global__ void __launch_bounds__(256, MINB) spmm_task_kernel(
     o = (uint32_t)it.w | ((__ldg(meta + t.z + lane) & kItemRMW) ? 0x80000000u : 0u);
   }
   if (t.x == t.y) {  // zero rows (build_tasks never mixes them with non-empty rows)
-    for (int r = 0; r < cnt; ++r) task_store(make_float4(0.f, 0.f, 0.f, 0.f), __shfl_sync(FULL, o, r), C, ldc, lane);
+    Frag<VEC> z;
+    z.zero();
+    for (int r = 0; r < cnt; ++r) task_store<VEC>(z, __shfl_sync(FULL, o, r), C, ldc);
     return;
   }
 #pragma unroll
@@ -379,29 +385,29 @@ __global__ void __launch_bounds__(256, MINB) spmm_task_kernel(
     const int v = __shfl_up_sync(FULL, end, d);
     if (lane >= d) end += v;
   }
-  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+  Frag<VEC> acc;
+  acc.zero();
   int r = 0;
   int row_end = t.x + __shfl_sync(FULL, end, 0);
   for (int eb = t.x; eb < t.y; eb += 32) {
     const int n = min(32, t.y - eb);
     const int2 my = lane < n ? __ldcs(ent + eb + lane) : make_int2(0, 0);
     for (int base = 0; base < n; base += U) {
-      float4 b[U];
+      Frag<VEC> b[U];
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         // past the end: re-load the last entry's row (same lines, no predicate, no zero fill)
         const int c = __shfl_sync(FULL, my.x, min(base + u, n - 1));
-        b[u] = __ldg(reinterpret_cast<const float4*>(reinterpret_cast<const char*>(Bk) + (uint64_t)(uint32_t)c * ldb));
+        b[u].load_g(reinterpret_cast<const float*>(reinterpret_cast<const char*>(Bk) + (uint64_t)(uint32_t)c * ldb));
       }
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         const float a = __int_as_float(__shfl_sync(FULL, my.y, base + u));
         if (base + u < n) {
-          acc.x = fmaf(a, b[u].x, acc.x); acc.y = fmaf(a, b[u].y, acc.y);
-          acc.z = fmaf(a, b[u].z, acc.z); acc.w = fmaf(a, b[u].w, acc.w);
+          acc.fma(a, b[u]);
           if (eb + base + u + 1 == row_end) {  // row r is complete (rows here are non-empty)
-            task_store(acc, __shfl_sync(FULL, o, r), C, ldc, lane);
-            acc = make_float4(0.f, 0.f, 0.f, 0.f);
+            task_store<VEC>(acc, __shfl_sync(FULL, o, r), C, ldc);
+            acc.zero();
             ++r;
             row_end = t.x + __shfl_sync(FULL, end, r & 31);
           }
@@ -1454,19 +1460,29 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
     const unsigned grid = (unsigned)((P.n_items + kSparseWarps - 1) / kSparseWarps);
     if (P.profiling) SR_TRY(prof_begin(P, 2, s));
     const int var = sparse_variant();
-    if (LPG == 32 && VEC == 4 && K % 128 == 0 && ldb * 4 < (1ll << 32) && var >= 4 && var <= 10 && P.n_tasks > 0) {
+    // row-group task kernels: K = 128·passes (float4 lanes) or 32·passes (float lanes)
+    const int tvec = (VEC == 4 && K % 128 == 0) ? 4 : (K % 32 == 0 && (var == 8 || var == 9) ? 1 : 0);
+    if (tvec && ldb * 4 < (1ll << 32) && var >= 4 && var <= 10 && P.n_tasks > 0) {
       const unsigned tgrid = (unsigned)((P.n_tasks + kSparseWarps - 1) / kSparseWarps);
+      const int pass = 32 * tvec;
       auto tk = [&](auto kern) {
-        for (int k0 = 0; k0 < K; k0 += 128)
+        for (int k0 = 0; k0 < K; k0 += pass)
           kern<<<tgrid, kSparseWarps * 32, 0, s>>>(P.tasks.p, P.n_tasks, P.items.p, P.item_meta.p, P.s_ent.p,
                                                     B + k0, (uint32_t)(ldb * 4), C + k0, ldc, (int)K, k0, P.scratch.p,
                                                     P.split_info.p, P.split_counter.p);
       };
-      switch (var) {
-        case 4: tk(spmm_task_kernel<4, 6>); break;
-        case 5: tk(spmm_task_kernel<8, 4>); break;
-        case 6: tk(spmm_task_kernel<2, 8>); break;
-        default: tk(spmm_task_kernel<4, 8>); break;
+      if (tvec == 4) {
+        switch (var) {
+          case 4: tk(spmm_task_kernel<4, 6, 4>); break;
+          case 5: tk(spmm_task_kernel<8, 4, 4>); break;
+          case 6: tk(spmm_task_kernel<2, 8, 4>); break;
+          default: tk(spmm_task_kernel<4, 8, 4>); break;
+        }
+      } else {
+        switch (var) {
+          case 9: tk(spmm_task_kernel<16, 4, 1>); break;
+          default: tk(spmm_task_kernel<8, 8, 1>); break;
+        }
       }
       SR_CUDA_TRY(cudaGetLastError());
       if (P.profiling) SR_TRY(prof_end(P, s));
