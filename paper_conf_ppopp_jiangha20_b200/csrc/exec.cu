@@ -1371,9 +1371,10 @@ int dense_engine() {  // 0 = coop, 1 = l1, 2 = tma
 }
 
 // Phase-S kernel choice (SR_SPARSE_VARIANT, measurement knob; profiles/r01/NOTES.md):
-// default = row-group task kernels (SpMM U 4 at 8 CTAs/SM, SDDMM U 2 at 4 CTAs/SM);
+// default (7) = row-group task kernels: SpMM K = 128·p float4 lanes U 4 at 8 CTAs/SM, SpMM
+// K = 32·p float lanes U 8 at 8 CTAs/SM, SDDMM K = 32·NCH <= 128 8-lane groups U 2 at 4 CTAs/SM;
 // 0 = one-row-per-warp kernels (U 2 / 8 CTAs); 1, 3 = row kernels at other occupancy points;
-// 4-7 = task kernels at other (U, CTAs/SM) points.
+// 4-6 = task kernels at other (U, CTAs/SM) points.
 int sparse_variant() {
   static const int v = [] {
     const char* d = getenv("SR_SPARSE_VARIANT");
@@ -1461,7 +1462,7 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
     if (P.profiling) SR_TRY(prof_begin(P, 2, s));
     const int var = sparse_variant();
     // row-group task kernels: K = 128·passes (float4 lanes) or 32·passes (float lanes)
-    const int tvec = (VEC == 4 && K % 128 == 0) ? 4 : (K % 32 == 0 && (var == 8 || var == 9) ? 1 : 0);
+    const int tvec = (VEC == 4 && K % 128 == 0) ? 4 : (K % 32 == 0 ? 1 : 0);
     if (tvec && ldb * 4 < (1ll << 32) && var >= 4 && var <= 10 && P.n_tasks > 0) {
       const unsigned tgrid = (unsigned)((P.n_tasks + kSparseWarps - 1) / kSparseWarps);
       const int pass = 32 * tvec;
@@ -1480,7 +1481,7 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
         }
       } else {
         switch (var) {
-          case 9: tk(spmm_task_kernel<16, 4, 1>); break;
+          case 5: tk(spmm_task_kernel<16, 4, 1>); break;
           default: tk(spmm_task_kernel<8, 8, 1>); break;
         }
       }
@@ -1564,8 +1565,6 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
       constexpr int NC = NCH > 4 ? 4 : NCH;  // (NCH <= 4 guarded above; keeps NCH 8 instantiable)
       switch (var) {
         case 4: tk(sddmm_task_kernel<NC, 2, 4>); break;
-        case 9: tk(sddmm_task_kernel<NC, 2, 5>); break;
-        case 10: tk(sddmm_task_kernel<NC, 4, 3>); break;
         case 5: tk(sddmm_task_kernel<NC, 1, 6>); break;
         case 6: tk(sddmm_task_kernel<NC, 1, 5>); break;
         default: tk(sddmm_task_kernel<NC, 2, 4>); break;
