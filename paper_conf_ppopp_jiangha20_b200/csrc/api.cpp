@@ -468,14 +468,14 @@ int check_params(const sr_reorder_params* p) {
 // LSH + Alg 3 over a column-sorted CSR (rows = the matrix being reordered).
 int reorder_round(const int64_t* rowptr, const int32_t* col, int64_t M, const sr_reorder_params& p,
                   cudaStream_t s, std::vector<int32_t>& perm, int64_t* E, double* t_lsh, double* t_cl) {
-  std::vector<uint64_t> pairs;
+  std::vector<uint64_t> pairs, by_key;
   std::vector<uint32_t> inter, uni;
   const double t0 = now_s();
-  SR_TRY(lsh_candidates(rowptr, col, M, rowptr[M], p, s, pairs, inter, uni, E));
+  SR_TRY(lsh_candidates(rowptr, col, M, rowptr[M], p, s, pairs, inter, uni, E, &by_key));
   const double t1 = now_s();
   perm.resize((size_t)M);
   cluster_rows(M, rowptr, col, (int64_t)pairs.size(), pairs.data(), inter.data(), uni.data(),
-               p.threshold_size, perm.data());
+               p.threshold_size, perm.data(), by_key.empty() ? nullptr : by_key.data());
   *t_lsh += t1 - t0;
   *t_cl += now_s() - t1;
   return SR_OK;
@@ -839,7 +839,7 @@ int sr_host_cluster(int64_t M, const int64_t* rowptr, const int32_t* colidx, int
     if (i >= j || (int64_t)j >= M || (e > 0 && pairs[e] <= pairs[e - 1]))
       return einval("sr_host_cluster: pairs must be sorted, unique, i < j < M");
   }
-  cluster_rows(M, rowptr, colidx, npairs, pairs, inter, uni, threshold_size, perm);
+  cluster_rows(M, rowptr, colidx, npairs, pairs, inter, uni, threshold_size, perm, pairs);  // key-sorted (checked)
   return SR_OK;
 }
 

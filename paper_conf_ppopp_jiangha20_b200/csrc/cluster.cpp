@@ -5,9 +5,11 @@
 // Library design (differs from the oracle's plain heap, same result):
 //  * the initial candidates arrive already sorted in heap order (J desc, then (i, j)
 //    asc; R10) from the GPU, so the initial heap is a read cursor over that array;
-//  * pairs re-inserted by Alg 3 line 28 go to a small binary heap; each pop takes the
-//    larger of the cursor head and the heap top under the same total order;
-//  * candidate-pair membership (line 27, R9) is an open-addressing hash set.
+//  * pairs re-inserted by Alg 3 line 28 go to an 8-ary heap; each pop takes the larger of
+//    the cursor head and the heap top under the same total order;
+//  * candidate-pair membership (line 27, R9): the initial candidates by binary search in the
+//    key-sorted pair array (the GPU's dedupe output), re-inserted pairs in an open-addressing
+//    hash set.  SR_DEBUG_CLUSTER=1 prints the phase times.
 // Readings R3-R12 decide everything the paper leaves open.
 #include <algorithm>
 #include <chrono>
@@ -16,7 +18,6 @@
 #include <parallel/algorithm>
 #include <cstring>
 #include <numeric>
-#include <queue>
 #include <vector>
 
 #include "internal.h"
@@ -37,8 +38,48 @@ inline bool before(const Cand& a, const Cand& b) {
   return a.j < b.j;
 }
 
-struct AfterCmp {  // std::priority_queue wants "less" = lower priority
-  bool operator()(const Cand& a, const Cand& b) const { return before(b, a); }
+// 8-ary max-heap under `before` (re-inserted pairs, Alg 3 line 28): log8 levels of one or two
+// cache lines each instead of log2 levels of one line — the heap can hold millions of pairs.
+// Its elements are distinct pairs under a strict total order, so the pop sequence is the same
+// as any other priority queue's.
+class DHeap {
+ public:
+  bool empty() const { return v_.empty(); }
+  const Cand& top() const { return v_[0]; }
+  void push(const Cand& c) {
+    size_t i = v_.size();
+    v_.push_back(c);
+    while (i > 0) {
+      const size_t p = (i - 1) / kD;
+      if (!before(c, v_[p])) break;
+      v_[i] = v_[p];
+      i = p;
+    }
+    v_[i] = c;
+  }
+  void pop() {
+    const Cand last = v_.back();
+    v_.pop_back();
+    const size_t n = v_.size();
+    if (n == 0) return;
+    size_t i = 0;
+    while (true) {
+      const size_t c0 = i * kD + 1;
+      if (c0 >= n) break;
+      size_t best = c0;
+      const size_t ce = std::min(n, c0 + kD);
+      for (size_t c = c0 + 1; c < ce; ++c)
+        if (before(v_[c], v_[best])) best = c;
+      if (!before(v_[best], last)) break;
+      v_[i] = v_[best];
+      i = best;
+    }
+    v_[i] = last;
+  }
+
+ private:
+  static constexpr size_t kD = 8;
+  std::vector<Cand> v_;
 };
 
 class PairSet {
@@ -135,14 +176,31 @@ inline void intersect(const int64_t* rowptr, const int32_t* col, int64_t a, int6
 
 void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t npairs,
                   const uint64_t* pairs, const uint32_t* inter, const uint32_t* uni,
-                  int32_t threshold_size, int32_t* perm) {
+                  int32_t threshold_size, int32_t* perm, const uint64_t* pairs_by_key) {
   const bool dbg = getenv("SR_DEBUG_CLUSTER") != nullptr;
   auto now = [] { return std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count(); };
   double t0 = now();
   // initial candidates in heap order; the membership set is built in parallel (the pairs are
   // distinct), the heap order is a strict total order (R10) so any sort gives the same array
   std::vector<Cand> init((size_t)npairs);
-  PairSet members((size_t)npairs + (size_t)npairs / 4);
+  // membership (line 27, R9): the initial candidates by binary search in their first row's
+  // segment of the key-sorted pair array (when the caller has it), re-inserted pairs in a hash
+  // set; without the key-sorted array every candidate goes into the hash set
+  const bool by_key = pairs_by_key != nullptr;
+  PairSet members(by_key ? (size_t)npairs / 4 + 16 : (size_t)npairs + (size_t)npairs / 4);
+  std::vector<int64_t> seg(by_key ? (size_t)M + 1 : 0);
+  if (by_key) {
+#pragma omp parallel for schedule(static)
+    for (int64_t r = 0; r <= M; ++r)
+      seg[r] = std::lower_bound(pairs_by_key, pairs_by_key + npairs, (uint64_t)r << 32) - pairs_by_key;
+  }
+  auto is_candidate = [&](uint64_t key) {
+    if (by_key) {
+      const int64_t lo = (int64_t)(key >> 32);
+      if (std::binary_search(pairs_by_key + seg[lo], pairs_by_key + seg[lo + 1], key)) return true;
+    }
+    return members.contains(key);
+  };
 #pragma omp parallel for schedule(static)
   for (int64_t e = 0; e < npairs; ++e) {
     Cand c;
@@ -156,15 +214,15 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
     }
     if (c.uni == 0) c.uni = 1;  // J(empty, empty) := 0/1 (R16)
     init[e] = c;
-    members.insert_distinct_concurrent(pairs[e]);
+    if (!by_key) members.insert_distinct_concurrent(pairs[e]);
   }
-  members.set_size((size_t)npairs);
+  if (!by_key) members.set_size((size_t)npairs);
   bool sorted = true;
   for (int64_t e = 1; e < npairs && sorted; ++e) sorted = !before(init[e], init[e - 1]);
   const double t1 = now();
   if (!sorted) __gnu_parallel::sort(init.begin(), init.end(), before);
   const double t2 = now();
-  int64_t n_reinsert = 0, n_pops = 0;
+  int64_t n_reinsert = 0;
 
   std::vector<int32_t> cid((size_t)M), csz((size_t)M, 1);
   std::vector<uint8_t> dead((size_t)M, 0);
@@ -176,7 +234,7 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
     }
     return x;
   };
-  std::priority_queue<Cand, std::vector<Cand>, AfterCmp> extra;
+  DHeap extra;
   size_t cur = 0;
   int64_t nclusters = M;
   while ((cur < init.size() || !extra.empty()) && nclusters > 0) {
@@ -206,7 +264,7 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
       if (dead[i] || dead[j] || i == j) continue;
       const uint32_t lo = (uint32_t)std::min(i, j), hi = (uint32_t)std::max(i, j);
       const uint64_t key = ((uint64_t)lo << 32) | hi;
-      if (members.contains(key)) continue;
+      if (is_candidate(key)) continue;
       Cand c;
       c.i = lo;
       c.j = hi;
@@ -220,7 +278,6 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
   if (dbg)
     fprintf(stderr, "cluster_rows: build %.3f s, sort %.3f s (sorted=%d), loop %.3f s, %lld re-inserted\n", t1 - t0,
             t2 - t1, (int)sorted, now() - t2, (long long)n_reinsert);
-  (void)n_pops;
   // rule B (R11): clusters of >= 2 rows by ascending root, then singletons ascending
   std::vector<int32_t> r_of((size_t)M);
   std::vector<int64_t> count((size_t)M + 1, 0);

@@ -205,13 +205,14 @@ void avgsim_positions(const Tiling& t, uint64_t* num, uint64_t* den);
 // cluster.cpp
 void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t npairs,
                   const uint64_t* pairs, const uint32_t* inter, const uint32_t* uni,
-                  int32_t threshold_size, int32_t* perm);
+                  int32_t threshold_size, int32_t* perm, const uint64_t* pairs_by_key = nullptr);
 void partition_panels(int64_t npanels, const int64_t* w, int32_t G, int64_t* cuts);
 // lsh.cu : device LSH candidate generation + exact Jaccard (sorted J order).
 // Returns candidate pairs sorted by (J desc, pair asc) with their (inter, uni).
 int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int64_t nnz,
                    const sr_reorder_params& p, cudaStream_t s, std::vector<uint64_t>& pairs_by_j,
-                   std::vector<uint32_t>& inter, std::vector<uint32_t>& uni, int64_t* E);
+                   std::vector<uint32_t>& inter, std::vector<uint32_t>& uni, int64_t* E,
+                   std::vector<uint64_t>* pairs_by_key = nullptr);
 // exec.cu : launchers
 int launch_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int64_t ldc,
                 cudaStream_t s, int32_t* launches);

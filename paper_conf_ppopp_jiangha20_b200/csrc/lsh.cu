@@ -213,7 +213,8 @@ inline unsigned blocks(int64_t n, int t) { return (unsigned)std::max<int64_t>(1,
 
 int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int64_t nnz,
                    const sr_reorder_params& p, cudaStream_t s, std::vector<uint64_t>& pairs_by_j,
-                   std::vector<uint32_t>& inter_h, std::vector<uint32_t>& uni_h, int64_t* E_out) {
+                   std::vector<uint32_t>& inter_h, std::vector<uint32_t>& uni_h, int64_t* E_out,
+                   std::vector<uint64_t>* pairs_by_key) {
   pairs_by_j.clear();
   inter_h.clear();
   uni_h.clear();
@@ -368,6 +369,10 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
   SR_CUDA_TRY(cudaMemcpyAsync(&E, nuniq.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
   SR_CUDA_TRY(cudaStreamSynchronize(s));
   sorted.release();
+  if (pairs_by_key) {  // the unique pairs in key order: the clustering's membership index (R9)
+    pairs_by_key->resize((size_t)E);
+    SR_CUDA_TRY(cudaMemcpyAsync(pairs_by_key->data(), allpairs.p, E * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+  }
   // exact Jaccard + heap-order sort
   DevBuf<uint32_t> d_inter, d_uni, idx_in, idx_out, i2, u2;
   DevBuf<uint64_t> jkey, jkey_out, p2;
