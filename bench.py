@@ -32,6 +32,7 @@ sys.path.insert(0, ROOT)
 
 from synth import generators as gen  # noqa: E402
 
+FP32_PEAK_GFLOPS = 148 * 128 * 2 * 1.965  # dense FP32 FMA peak (74.4 TFLOP/s), DESIGN.md §5
 PAPER_CONTEXT = ("P100 (paper, P:334, P:350): ASpT-RR up to 2.91x SpMM vs best of ASpT-NR/cuSPARSE and "
                  "up to 3.19x SDDMM vs ASpT-NR; geomean 1.19x / 1.49x (K=1024)")
 
@@ -356,6 +357,9 @@ def run_ours(args, A, ops, rank, world, local_rank):
                 if rec is not None:
                     dk["dram_bytes_ncu"] = rec["bytes"]
                     dk["dram_gbs"] = rec["bytes"] / (dk["avg_ms"] / 1e3) / 1e9
+                    for hk in ("l2_hit_pct", "l1_hit_pct"):
+                        if hk in rec:
+                            dk[hk + "_ncu"] = rec[hk]
 
     # the same kernel against the L2 -> SM gather ceiling (the path every gathered row takes;
     # DESIGN.md §5): a conservative efficiency for a gather-bound kernel whose HBM bytes are
@@ -480,7 +484,9 @@ def run_ours(args, A, ops, rank, world, local_rank):
             ks = [k for k in kern if k.startswith(name)]
             if ks:
                 ms = sum(kern[k]["avg_ms"] for k in ks)
-                per_op[name] = {"ms": ms, "gflops": 2.0 * A.nnz * K / (ms / 1e3) / 1e9 if world == 1 else None}
+                gf = 2.0 * A.nnz * K / (ms / 1e3) / 1e9 if world == 1 else None
+                # FP32 fraction: against 148 SMs x 128 FP32 lanes x 2 x 1.965 GHz
+                per_op[name] = {"ms": ms, "gflops": gf, "fp32_frac": gf / FP32_PEAK_GFLOPS if gf else None}
         line["per_op_gflops"] = per_op
         print(json.dumps(line), flush=True)
 

@@ -32,7 +32,11 @@ def main(path, config, K, tag=""):
             total += float(d[ix[m]]) * UNIT[units[ix[m]]]
         t = float(d[ix["gpu__time_duration.sum"]]) * {"nsecond": 1e-9, "ns": 1e-9, "usecond": 1e-6, "us": 1e-6,
                                                        "msecond": 1e-3, "ms": 1e-3}[units[ix["gpu__time_duration.sum"]]]
-        table[f"{config}_K{K}_{kind}"] = {"bytes": total, "ncu_duration_s": t, "source": tag or os.path.basename(path)}
+        rec = {"bytes": total, "ncu_duration_s": t, "source": tag or os.path.basename(path)}
+        for m, key in (("lts__t_sector_hit_rate.pct", "l2_hit_pct"), ("l1tex__t_sector_hit_rate.pct", "l1_hit_pct")):
+            if m in ix and d[ix[m]] not in ("", "n/a"):
+                rec[key] = float(d[ix[m]])
+        table[f"{config}_K{K}_{kind}"] = rec
     json.dump(table, open(out_path, "w"), indent=1, sort_keys=True)
     print(json.dumps(table, indent=1))
 

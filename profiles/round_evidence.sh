@@ -12,3 +12,4 @@ timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/$
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${tag}_launches.csv \
   python bench.py --steps 2 --warmup 1 --min-warm-s 0 --e2e-steps 0 --no-cpu-baseline > /dev/null 2>&1; echo "launches rc=$?"
 timeout 900 bash profiles/ncu_capture.sh ${tag}k128 "spmm_task|sddmm_task|spmm_dense|sddmm_dense" 4 > /dev/null 2>&1; echo "ncu k128 rc=$?"
+timeout 900 bash profiles/ncu_capture.sh ${tag}k32 "spmm_task|sddmm_task|spmm_dense|sddmm_dense" 4 --K 32 > /dev/null 2>&1; echo "ncu k32 rc=$?"
