@@ -431,7 +431,9 @@ __device__ __forceinline__ void cp_async_cg16(void* dst, const void* src) {
 }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
 
-template <int NCH, int U, int MINB>
+// PERM: lane 8g+k holds batch entry 4k+g, so in step s group g's entry (4s+g) sits in its own
+// lane 8g+s, which stores the result from its own registers (no value / index shuffles).
+template <int NCH, int U, int MINB, bool PERM = false>
 __global__ void __launch_bounds__(256, MINB) sddmm_task_kernel(
     const int4* __restrict__ tasks, int64_t n_tasks, const Item* __restrict__ items, const int2* __restrict__ ent,
     const int32_t* __restrict__ oidx, const float* __restrict__ X, int64_t ldx, const float* __restrict__ Y,
@@ -468,10 +470,11 @@ __global__ void __launch_bounds__(256, MINB) sddmm_task_kernel(
   bool staged = false;
   for (int eb = t.x; eb < t.y; eb += 32) {
     const int n = min(32, t.y - eb);
-    const int2 my = lane < n ? __ldcs(ent + eb + lane) : make_int2(0, 0);
-    const int myo = lane < n ? __ldcs(oidx + eb + lane) : 0;
+    const int me = PERM ? 4 * lg + g : lane;  // batch entry this lane loads
+    const int2 my = me < n ? __ldcs(ent + eb + me) : make_int2(0, 0);
+    const int myo = me < n ? __ldcs(oidx + eb + me) : 0;
     // row (within the task) of the entry this lane loaded
-    const int rel = eb + lane - t.x;
+    const int rel = eb + me - t.x;
     int myrow = 0;
     for (int r = 0; r < cnt; ++r) myrow += (__shfl_sync(FULL, end, r) <= rel) ? 1 : 0;
     if (!staged) {
@@ -485,8 +488,9 @@ __global__ void __launch_bounds__(256, MINB) sddmm_task_kernel(
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         const int jj = min(base + u * G + g, n - 1);
-        const int c = __shfl_sync(FULL, my.x, jj);
-        row[u] = __shfl_sync(FULL, myrow, jj);
+        const int src = PERM ? (((jj & 3) << 3) | (jj >> 2)) : jj;
+        const int c = __shfl_sync(FULL, my.x, src);
+        row[u] = __shfl_sync(FULL, myrow, src);
         const char* yp = Yl + (uint64_t)(uint32_t)c * ldy_bytes;
 #pragma unroll
         for (int ch = 0; ch < NCH; ++ch) y[u][ch] = __ldg(reinterpret_cast<const float4*>(yp + ch * 128));
@@ -513,9 +517,13 @@ __global__ void __launch_bounds__(256, MINB) sddmm_task_kernel(
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         const int j = base + u * G + g;
-        const float v = __int_as_float(__shfl_sync(FULL, my.y, j & 31));
-        const int o = __shfl_sync(FULL, myo, j & 31);
-        if (lg == 0 && j < n) __stcs(out + o, v * part[u]);
+        if (PERM) {
+          if (lg == (j >> 2) && j < n) __stcs(out + myo, __int_as_float(my.y) * part[u]);
+        } else {
+          const float v = __int_as_float(__shfl_sync(FULL, my.y, j & 31));
+          const int o = __shfl_sync(FULL, myo, j & 31);
+          if (lg == 0 && j < n) __stcs(out + o, v * part[u]);
+        }
       }
     }
   }
@@ -1565,6 +1573,7 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
       constexpr int NC = NCH > 4 ? 4 : NCH;  // (NCH <= 4 guarded above; keeps NCH 8 instantiable)
       switch (var) {
         case 4: tk(sddmm_task_kernel<NC, 2, 4>); break;
+        case 8: tk(sddmm_task_kernel<NC, 2, 4, true>); break;
         case 5: tk(sddmm_task_kernel<NC, 1, 6>); break;
         case 6: tk(sddmm_task_kernel<NC, 1, 5>); break;
         default: tk(sddmm_task_kernel<NC, 2, 4>); break;
