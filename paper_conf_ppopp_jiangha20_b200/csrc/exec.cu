@@ -1380,7 +1380,8 @@ int dense_engine() {  // 0 = coop, 1 = l1, 2 = tma
 
 // Phase-S kernel choice (SR_SPARSE_VARIANT, measurement knob; profiles/r01/NOTES.md):
 // default (7) = row-group task kernels: SpMM K = 128·p float4 lanes U 4 at 8 CTAs/SM, SpMM
-// K = 32·p float lanes U 8 at 8 CTAs/SM, SDDMM K = 32·NCH <= 128 8-lane groups U 2 at 4 CTAs/SM;
+// K = 32·p float lanes U 8 at 8 CTAs/SM, SDDMM K = 32·NCH <= 128 8-lane groups U 2 at 4 CTAs/SM
+// with the permuted entry layout (4 = lane-order layout);
 // 0 = one-row-per-warp kernels (U 2 / 8 CTAs); 1, 3 = row kernels at other occupancy points;
 // 4-6 = task kernels at other (U, CTAs/SM) points.
 int sparse_variant() {
@@ -1572,11 +1573,9 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
       };
       constexpr int NC = NCH > 4 ? 4 : NCH;  // (NCH <= 4 guarded above; keeps NCH 8 instantiable)
       switch (var) {
-        case 4: tk(sddmm_task_kernel<NC, 2, 4>); break;
-        case 8: tk(sddmm_task_kernel<NC, 2, 4, true>); break;
-        case 5: tk(sddmm_task_kernel<NC, 1, 6>); break;
-        case 6: tk(sddmm_task_kernel<NC, 1, 5>); break;
-        default: tk(sddmm_task_kernel<NC, 2, 4>); break;
+        case 4: tk(sddmm_task_kernel<NC, 2, 4>); break;  // entries in lane order (shuffled values)
+        case 5: tk(sddmm_task_kernel<NC, 1, 6, true>); break;
+        default: tk(sddmm_task_kernel<NC, 2, 4, true>); break;
       }
       SR_CUDA_TRY(cudaGetLastError());
       if (P.profiling) SR_TRY(prof_end(P, s));
