@@ -154,9 +154,28 @@ def cpu_baseline(A, K, args, ops, name):
         if "sddmm" in ops:
             O.sddmm(s["sub"], s["X"], s["Y"])
     dt = time.perf_counter() - t0
-    return {"value": s["flops"] * reps / dt / 1e9, "unit": "GFLOP/s", "cores": O.num_threads(), "kind": "oracle",
+    cores = O.num_threads()
+    # single-thread leg (O1/O2 timed single-thread and on all cores), on a
+    # 1/cores share of the sample's rows so it stays within the same time budget
+    R1 = max(1, s["rows"] // max(cores, 1))
+    sub1 = gen.CSR(R1, A.ncols, A.rowptr[:R1 + 1].copy(), A.colidx[:A.rowptr[R1]], A.vals[:A.rowptr[R1]])
+    X1 = s["X"][:R1] if s["X"] is not None else None
+    O.set_num_threads(1)
+    try:
+        t1 = time.perf_counter()
+        if "spmm" in ops:
+            O.spmm(sub1, s["B"])
+        if "sddmm" in ops:
+            O.sddmm(sub1, X1, s["Y"])
+        dt1 = time.perf_counter() - t1
+    finally:
+        O.set_num_threads(cores)
+    st_value = 2.0 * int(sub1.rowptr[-1]) * K * len(ops) / max(dt1, 1e-9) / 1e9
+    return {"value": s["flops"] * reps / dt / 1e9, "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
             "sample": f"{name} rows [0,{s['rows']}) = {s['nnz']} nnz of {A.nnz}, K={K}, {'+'.join(ops)} in fp64, "
-                      f"{reps} pass(es), {dt:.1f} s"}
+                      f"{reps} pass(es), {dt:.1f} s",
+            "single_thread": {"value": st_value, "unit": "GFLOP/s", "cores": 1,
+                              "sample": f"rows [0,{R1}) = {int(sub1.rowptr[-1])} nnz, {dt1:.1f} s"}}
 
 
 def run_reference(args, A, ops, rank, world):

@@ -59,6 +59,7 @@ def lib():
             "or_partition": (None, [i64, P, i32, P]),
             "or_access_count": (i64, [i64, P, P, P, i64, P, i32]),
             "or_num_threads": (C.c_int, []),
+            "or_set_num_threads": (None, [C.c_int]),
         }
         for name, (res, args) in sig.items():
             f = getattr(_lib, name)
@@ -77,6 +78,11 @@ def _c(a, dtype):
 
 def num_threads() -> int:
     return lib().or_num_threads()
+
+
+def set_num_threads(n: int) -> None:
+    """OpenMP threads of the oracle's parallel loops (timing legs only; results unchanged)."""
+    lib().or_set_num_threads(int(n))
 
 
 # ---------------------------------------------------------------- O0 .. O2
