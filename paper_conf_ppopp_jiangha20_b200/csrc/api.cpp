@@ -110,7 +110,7 @@ void sparse_traffic(const ItemBuilder& ib, int64_t n_nonzero, int64_t n_zero, co
 int32_t task_nnz() {
   static const int32_t v = [] {
     const char* e = getenv("SR_TASK_NNZ");
-    const int x = e ? atoi(e) : 128;  // measured best of 32/64/128/256 on C2 (profiles/r01/NOTES.md)
+    const int x = e ? atoi(e) : 256;  // measured best of 64..1024 on C2 (profiles/r01/tasknnz, NOTES.md)
     return x < 1 ? 1 : x;
   }();
   return v;

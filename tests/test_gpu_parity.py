@@ -360,7 +360,7 @@ def test_dist_gather_single_rank_nccl(env, oracle):
 @pytest.mark.parametrize("var,val", [("SR_DENSE_ENGINE", "coop"), ("SR_DENSE_ENGINE", "l1"),
                                      ("SR_SPARSE_VARIANT", "0"), ("SR_SPARSE_VARIANT", "4"),
                                      ("SR_SPARSE_VARIANT", "5"),
-                                     ("SR_TASK_NNZ", "1")])
+                                     ("SR_TASK_NNZ", "1"), ("SR_TASK_NNZ", "1024")])
 def test_engines_subprocess(env, var, val):
     """The phase-D engine (SR_DENSE_ENGINE) and the phase-S kernels (SR_SPARSE_VARIANT: 0 =
     one-row-per-warp kernels, 4, 5 = task kernels at other occupancy points / entry layouts; SR_TASK_NNZ=1 = one
