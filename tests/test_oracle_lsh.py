@@ -208,3 +208,34 @@ def test_jaccard_matches_python_sets(oracle):
     for e, key in enumerate(pairs.tolist()):
         i, j = key >> 32, key & MASK32
         assert inter[e] == len(rows[i] & rows[j]) and uni[e] == len(rows[i] | rows[j])
+
+
+def _splitmix64_py(seed: int, n: int):
+    """SplitMix64 (Steele, Lea & Flood 2014) written out in Python, independent of the oracle."""
+    M64 = (1 << 64) - 1
+    s, out = seed & M64, []
+    for _ in range(n):
+        s = (s + 0x9E3779B97F4A7C15) & M64
+        z = s
+        z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & M64
+        z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & M64
+        out.append(z ^ (z >> 31))
+    return out
+
+
+def test_python_splitmix64_matches_published_vector():
+    assert _splitmix64_py(1234567, 5) == [
+        6457827717110365317, 3203168211198807973, 9817491932198370423,
+        4593380528125082431, 16408922859458223821]
+
+
+@pytest.mark.parametrize("seed,siglen", [(4, 128), (0, 7), (2 ** 63 + 5, 33)])
+def test_hash_params_draw_order(oracle, seed, siglen):
+    """R13 (O3): for s = 0..siglen-1 in order, a_s = (next() & 0xFFFFFFFF) | 1 and then
+    b_s = next() & 0xFFFFFFFF from one SplitMix64 stream seeded with `seed`; i.e. draw 2s
+    is a_s's and draw 2s+1 is b_s's.  A swapped (a, b) draw order or a per-array stream
+    fails here."""
+    st = _splitmix64_py(seed, 2 * siglen)
+    a, b = oracle.hash_params(seed, siglen)
+    assert a.tolist() == [(st[2 * s] & MASK32) | 1 for s in range(siglen)]
+    assert b.tolist() == [st[2 * s + 1] & MASK32 for s in range(siglen)]

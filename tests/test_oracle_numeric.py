@@ -122,3 +122,18 @@ def test_canonicalize_rejects_bad_input(oracle):
     bad.rowptr[2] = 1  # decreasing
     with pytest.raises(ValueError):
         oracle.canonicalize(bad)
+
+
+@pytest.mark.parametrize("M,N,dens,empty,seed", CASES)
+@pytest.mark.parametrize("K", [1, 7, 16])
+def test_sddmm_bound_scale_elementwise(oracle, M, N, dens, empty, seed, K):
+    """The tolerance scale of every GPU SDDMM check (north_star: |err| <= 1e-4·Σ|a||x||y|)
+    is out_abs[p] = |a_ij|·Σ_k |x_ik|·|y_jk|: pinned element by element against numpy's
+    (|X| @ |Y|ᵀ) ⊙ |A| in fp64, not only as an upper bound of |out|."""
+    A = g.random_csr(M, N, dens, seed, empty_frac=empty)
+    X = g.dense(M, K, seed=seed, stream=1)
+    Y = g.dense(N, K, seed=seed, stream=2)
+    full = (np.abs(X.astype(np.float64)) @ np.abs(Y.astype(np.float64)).T) * np.abs(dense_of(A))
+    r = np.repeat(np.arange(A.nrows), np.diff(A.rowptr))
+    _, gabs = oracle.sddmm(A, X, Y)
+    np.testing.assert_allclose(gabs, full[r, A.colidx], rtol=1e-12, atol=0)

@@ -73,6 +73,27 @@ def test_larger_cluster_wins_and_tie_goes_to_smaller_index(oracle):
     assert perm.tolist() == [2, 3, 4, 0, 1]
 
 
+def test_equal_size_root_is_smaller_index_output_order(oracle):
+    """R6 (Fig 6 first merge (0,4) -> root 0) seen through rule B's root order:
+    pairs (0,3) and (1,2), both J = 1, equal sizes.  Smaller-index roots 0 and 1 ->
+    clusters emitted as [0,3] then [1,2]; larger-index roots (3 and 2) would emit [1,2]
+    first (hand-derived)."""
+    A = _csr([{1}, {2}, {2}, {1}], 4)
+    perm = oracle.cluster(A.rowptr, A.colidx, oracle.pack_pairs([(0, 3), (1, 2)]), 256)
+    assert perm.tolist() == [0, 3, 1, 2]
+
+
+def test_size_update_drives_threshold_deletion(oracle):
+    """R4 + R7: after merging (0,1) the cluster has size 2 >= threshold 2 and is
+    deleted, so the later pair (1,3) (root 0 deleted) is skipped and row 3 stays a singleton:
+    [0,1,2,3].  Without the size update the cluster would absorb row 3 through the
+    re-inserted pair (0,3) (J = 2/3) and give [0,1,3,2] (hand-derived)."""
+    A = _csr([{1, 2}, {1, 2}, {7}, {1, 2, 3}], 8)
+    perm = oracle.cluster(A.rowptr, A.colidx, oracle.pack_pairs([(0, 1), (1, 3)]), 2)
+    assert perm.tolist() == [0, 1, 2, 3]
+    assert oracle.cluster(A.rowptr, A.colidx, oracle.pack_pairs([(0, 1), (1, 3)]), 256).tolist() == [0, 1, 3, 2]
+
+
 def _check_invariants(perm, M, threshold):
     assert sorted(perm.tolist()) == list(range(M))
 
@@ -204,6 +225,55 @@ def test_auto_runs_round1_on_scattered_matrix(oracle):
     assert p["stats"]["dense0"] * 10 <= p["stats"]["nnz"]
     assert p["stats"]["round1"] == 1
     assert sorted(p["perm1"].tolist()) == list(range(512))
+
+
+def test_auto_on_fig1a_skips_round1_runs_round2(oracle):
+    """Fig 1a under AUTO with the example's ASpT parameters (panel 3, dense >= 2):
+    DenseRatio0 = 2/13 > 1/10 -> round 1 skipped, perm1 = identity.  The
+    remainder of the identity tiling is {0}, {1,2,3}, {5} | {1}, {0,3,4}, {2,5} (column 4 of
+    panel 0 is the only dense column): no two consecutive rows share a column, so
+    AvgSim = 0 <= 1/10 and round 2 runs (hand-derived)."""
+    A = g.fig1a()
+    p = oracle.plan(A, panel_rows=3, dense_min=2, mode=oracle.MODE_AUTO)
+    st = p["stats"]
+    assert (st["dense0"], st["nnz"]) == (2, 13)
+    assert st["round1"] == 0 and p["perm1"].tolist() == list(range(6))
+    assert st["avgsim_num"] == 0 and st["round2"] == 1
+    assert sorted(p["perm2"].tolist()) == list(range(6))
+
+
+def test_auto_skips_round2_when_remainder_is_clustered(oracle):
+    """skip round 2 iff AvgSim > 0.1.  Rows {0,1},{0,1},{5,6},{5,6}, no dense
+    columns (dense_min 100): DenseRatio0 = 0 -> round 1 runs; LSH pairs the identical
+    rows (every band collides), Alg 3 keeps perm1 = [0,1,2,3]; AvgSim = (1+0+1)/3 = 2/3
+    > 1/10 -> round 2 skipped, perm2 = [0,1,2,3], E2 = 0 (hand-derived)."""
+    A = _csr([{0, 1}, {0, 1}, {5, 6}, {5, 6}], 8)
+    p = oracle.plan(A, panel_rows=2, dense_min=100, mode=oracle.MODE_AUTO)
+    st = p["stats"]
+    assert st["round1"] == 1 and p["perm1"].tolist() == [0, 1, 2, 3]
+    assert st["avgsim_num"] * 3 == st["avgsim_den"] * 2
+    assert st["round2"] == 0 and st["E2"] == 0 and p["perm2"].tolist() == [0, 1, 2, 3]
+
+
+@pytest.mark.parametrize("pairs,expect_round2", [(1, 1), (2, 0)])
+def test_auto_round2_threshold_is_strict(oracle, pairs, expect_round2):
+    """"greater than 0.1" (R20 strict >).  11 non-empty rows with one identical
+    pair (rows 0, 5): round 1 clusters them (rule B: [0, 5, 1, 2, 3, 4, 6, ...]) and the
+    remainder's AvgSim is exactly 1/10 -> round 2 runs.  12 rows with two identical
+    pairs (0, 5) and (6, 11): AvgSim = 2/11 > 1/10 -> round 2 skipped."""
+    n = 11 if pairs == 1 else 12
+    sets = [{20 + i} for i in range(n)]
+    sets[0] = sets[5] = {0, 1}
+    if pairs == 2:
+        sets[6] = sets[11] = {2, 3}
+    A = _csr(sets, 40)
+    p = oracle.plan(A, panel_rows=4, dense_min=100, mode=oracle.MODE_AUTO)
+    st = p["stats"]
+    clustered = [0, 5] if pairs == 1 else [0, 5, 6, 11]
+    expect1 = clustered + [r for r in range(n) if r not in clustered]
+    assert st["round1"] == 1 and p["perm1"].tolist() == expect1
+    assert st["avgsim_num"] * (n - 1) == st["avgsim_den"] * pairs
+    assert st["round2"] == expect_round2
 
 
 def test_plan_modes_consistent(oracle):
