@@ -72,17 +72,28 @@ typedef struct {
   int32_t skip_dense_num, skip_dense_den; /* skip round 1 iff DenseRatio0 > num/den (1/10) */
   int32_t skip_sim_num, skip_sim_den;     /* skip round 2 iff AvgSim > num/den (1/10)      */
   int32_t world, rank;     /* row-panel shard owned by this handle; 1, 0 = whole matrix    */
+  int32_t auto_dense_min;  /* dense criterion of the AUTO DenseRatio0 decision (R28);
+                              0 = dense_min.  Lets the decision ask "does the original order
+                              already share columns?" while the kernels run with a higher
+                              execution threshold                           */
+  int32_t reserved0;       /* must be 0                                                    */
 } sr_reorder_params;
 
 /* Fill *p with the defaults above (siglen 128, bsize 2, threshold 256, max_bucket 32,
- * seed 4, panel_rows 64, dense_min 2, tile_cols 64, AUTO, 1/10, 1/10, world 1, rank 0). */
+ * seed 4, panel_rows 64, dense_min 2, tile_cols 64, AUTO, 1/10, 1/10, world 1, rank 0,
+ * auto_dense_min 0). */
 void sr_default_params(sr_reorder_params* p);
+
+/* The parameters of h's plan (after sr_reorder or sr_plan_load; the defaults before).
+ * Errors: SR_EINVAL (NULL). */
+int sr_get_params(sr_csr h, sr_reorder_params* out);
 
 /* -----------------------------------------------------------------------------
  * sr_reorder — build the plan (Fig 5 workflow):
  *   round 1: LSH candidate pairs of A's rows (minhash + banding on the GPU,
  *            P:151-153) -> exact Jaccard (GPU) -> Alg 3 clustering (host,
- *            P:155-222) -> perm1;  skipped under AUTO if DenseRatio0 > 1/10.
+ *            P:155-222) -> perm1;  skipped under AUTO if DenseRatio0 > 1/10
+ *            (DenseRatio0 with the dense criterion auto_dense_min, R28).
  *   ASpT tiling of perm1's row panels: dense columns + remainder.
  *   round 2: the same on the remainder rows -> perm2; skipped under AUTO if the
  *            remainder's consecutive-row AvgSim > 1/10.
@@ -186,7 +197,8 @@ int sr_get_perm(sr_csr h, int which, int32_t* out, int64_t cap, int64_t* len);
 
 typedef struct {
   int64_t nnz;
-  int64_t dense0;        /* dense-tile nnz of the original order: DenseRatio0 = dense0/nnz */
+  int64_t dense0;        /* dense-tile nnz of the original order under the AUTO decision's
+                            criterion (auto_dense_min, else dense_min): DenseRatio0 = dense0/nnz */
   int64_t dense1;        /* dense-tile nnz of the plan:           DenseRatio  = dense1/nnz */
   uint64_t avgsim_num;   /* AvgSim of the remainder = num/den (R27 fixed point)          */
   uint64_t avgsim_den;

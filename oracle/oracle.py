@@ -54,7 +54,7 @@ def lib():
             "or_reorder_rows": (i64, [i64, P, P, i32, i32, u64, i32, i32, P]),
             "or_tile": (i64, [i64, i64, P, P, P, i32, i32, P, P, P, P, P, P, P, P]),
             "or_avgsim": (u64, [i64, P, P, P]),
-            "or_plan": (C.c_int, [i64, i64, P, P, i32, i32, u64, i32, i32, i32, i32, i32, i32,
+            "or_plan": (C.c_int, [i64, i64, P, P, i32, i32, u64, i32, i32, i32, i32, i32, i32, i32,
                                   i32, i32, i32, P, P, P, P, P, P, P, P, P, P, P, P]),
             "or_partition": (None, [i64, P, i32, P]),
             "or_access_count": (i64, [i64, P, P, P, i64, P, i32]),
@@ -255,7 +255,7 @@ STAT_KEYS = ("dense0", "dense1", "nnz", "avgsim_num", "avgsim_den", "round1", "r
 
 
 def plan(A, siglen=128, bsize=2, seed=4, max_bucket=0, threshold_size=256, panel_rows=64,
-         dense_min=2, mode=MODE_AUTO, skip_dense=(1, 10), skip_sim=(1, 10)) -> dict:
+         dense_min=2, mode=MODE_AUTO, skip_dense=(1, 10), skip_sim=(1, 10), auto_dense_min=0) -> dict:
     M, N, nnz = A.nrows, A.ncols, A.nnz
     rp, ci = _c(A.rowptr, np.int64), _c(A.colidx, np.int32)
     npan = (M + panel_rows - 1) // panel_rows
@@ -268,7 +268,7 @@ def plan(A, siglen=128, bsize=2, seed=4, max_bucket=0, threshold_size=256, panel
              d_pos=np.zeros(max(nnz, 1), np.int64), rrow_ptr=np.zeros(M + 1, np.int64),
              r_col=np.zeros(max(nnz, 1), np.int32), r_pos=np.zeros(max(nnz, 1), np.int64))
     rc = lib().or_plan(M, N, _p(rp), _p(ci), siglen, bsize, seed, max_bucket, threshold_size,
-                       panel_rows, dense_min, mode, skip_dense[0], skip_dense[1], skip_sim[0],
+                       panel_rows, dense_min, auto_dense_min, mode, skip_dense[0], skip_dense[1], skip_sim[0],
                        skip_sim[1], _p(perm1), _p(perm2), C.byref(n2),
                        *[_p(t[k]) for k in ("dense_ptr", "dense_cols", "drow_ptr", "d_slot", "d_pos",
                                             "rrow_ptr", "r_col", "r_pos")], _p(stats))

@@ -33,7 +33,11 @@ class ReorderParams(C.Structure):
                 ("dense_min", C.c_int32), ("tile_cols", C.c_int32), ("mode", C.c_int32),
                 ("skip_dense_num", C.c_int32), ("skip_dense_den", C.c_int32),
                 ("skip_sim_num", C.c_int32), ("skip_sim_den", C.c_int32),
-                ("world", C.c_int32), ("rank", C.c_int32)]
+                ("world", C.c_int32), ("rank", C.c_int32), ("auto_dense_min", C.c_int32),
+                ("reserved0", C.c_int32)]
+
+    def as_dict(self) -> dict:
+        return {k: getattr(self, k) for k, _ in self._fields_}
 
 
 class PlanStats(C.Structure):
@@ -65,7 +69,7 @@ EXPORTED = ("sr_csr_create", "sr_default_params", "sr_reorder", "sr_spmm", "sr_s
             "sr_get_perm", "sr_get_plan_stats", "sr_export_tiles", "sr_shard_rows", "sr_shard_nnz_ids",
             "sr_last_launch_count", "sr_last_error", "sr_host_cluster", "sr_host_partition", "sr_version",
             "sr_get_traffic_model", "sr_set_profiling", "sr_last_kernel_times", "sr_scatter_rows",
-            "sr_scatter_values", "sr_plan_save", "sr_plan_load", "sr_trial", "sr_set_values")
+            "sr_scatter_values", "sr_plan_save", "sr_plan_load", "sr_trial", "sr_set_values", "sr_get_params")
 
 _lib = None
 
@@ -88,6 +92,7 @@ def lib():
         "sr_destroy": (C.c_int, [P]),
         "sr_get_perm": (C.c_int, [P, C.c_int, P, i64, C.POINTER(i64)]),
         "sr_get_plan_stats": (C.c_int, [P, C.POINTER(PlanStats)]),
+        "sr_get_params": (C.c_int, [P, C.POINTER(ReorderParams)]),
         "sr_export_tiles": (C.c_int, [P] + [P] * 8),
         "sr_shard_rows": (C.c_int, [P, P, i64, C.POINTER(i64)]),
         "sr_shard_nnz_ids": (C.c_int, [P, P, i64, C.POINTER(i64)]),
@@ -204,11 +209,14 @@ class SparseMatrix:
         s = C.c_void_p(int(stream.cuda_stream)) if stream is not None else C.c_void_p()
         buf = C.create_string_buffer(bytes(image), len(image))
         _check(lib().sr_plan_load(self._h, C.cast(buf, C.c_void_p), len(image), world, rank, s))
-        p = ReorderParams()
-        lib().sr_default_params(C.byref(p))
-        p.world, p.rank = world, rank
-        self.params = p
+        self.params = self.get_params()
         return self.stats()
+
+    def get_params(self) -> ReorderParams:
+        """The parameters of this handle's plan (sr_get_params)."""
+        p = ReorderParams()
+        _check(lib().sr_get_params(self._h, C.byref(p)))
+        return p
 
     def stats(self) -> dict:
         st = PlanStats()

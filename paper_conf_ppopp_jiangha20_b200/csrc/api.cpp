@@ -462,6 +462,8 @@ int check_params(const sr_reorder_params* p) {
   if (p->skip_dense_den <= 0 || p->skip_sim_den <= 0 || p->skip_dense_num < 0 || p->skip_sim_num < 0)
     return einval("decision thresholds must be non-negative fractions");
   if (p->world < 1 || p->rank < 0 || p->rank >= p->world) return einval("bad world / rank");
+  if (p->auto_dense_min < 0) return einval("auto_dense_min must be >= 0 (0 = dense_min)");
+  if (p->reserved0 != 0) return einval("reserved0 must be 0");
   return SR_OK;
 }
 
@@ -648,11 +650,13 @@ int sr_reorder(sr_csr h, const sr_reorder_params* p, sr_stream stream) {
   st.nnz = nnz;
   std::vector<int32_t> ident((size_t)M);
   std::iota(ident.begin(), ident.end(), 0);
-  // DenseRatio of the original order
+  // DenseRatio of the original order under the decision's dense criterion (R28)
   double t0 = now_s();
+  const int32_t dense_min0 = p->auto_dense_min > 0 ? p->auto_dense_min : p->dense_min;
   Tiling t_id;
-  tile_rows(A, ident, p->panel_rows, p->dense_min, t_id);
+  tile_rows(A, ident, p->panel_rows, dense_min0, t_id);
   st.dense0 = t_id.n_dense();
+  if (dense_min0 != p->dense_min) tile_rows(A, ident, p->panel_rows, p->dense_min, t_id);
   st.t_tile_s += now_s() - t0;
   bool round1 = p->mode == SR_REORDER_FORCE;
   if (p->mode == SR_REORDER_AUTO)
@@ -737,6 +741,12 @@ int sr_get_perm(sr_csr h, int which, int32_t* out, int64_t cap, int64_t* len) {
   *len = (int64_t)v->size();
   if (cap < *len) return out ? einval("sr_get_perm: capacity too small") : SR_OK;
   if (out && !v->empty()) std::memcpy(out, v->data(), v->size() * sizeof(int32_t));
+  return SR_OK;
+}
+
+int sr_get_params(sr_csr h, sr_reorder_params* out) {
+  if (!h || !out) return einval("sr_get_params: NULL argument");
+  *out = h->params;
   return SR_OK;
 }
 
@@ -867,7 +877,7 @@ int sr_host_partition(int64_t npanels, const int64_t* weights, int32_t G, int64_
 namespace sr {
 namespace {
 constexpr char kPlanMagic[8] = {'S', 'R', 'P', 'L', 'A', 'N', '0', '1'};
-constexpr uint32_t kPlanVersion = 1;
+constexpr uint32_t kPlanVersion = 2;  // 2: sr_reorder_params gained auto_dense_min
 
 // 64-bit hash of a byte range (word-wise multiply-xorshift; not cryptographic).
 uint64_t hash_bytes(const void* p, size_t n, uint64_t h) {

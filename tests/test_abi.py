@@ -33,14 +33,40 @@ def test_exports_every_declared_symbol(sr):
     assert declared == set(sr.EXPORTED)
 
 
-def test_struct_layouts_match_header(sr):
-    # sr_reorder_params: 4 int32, u64 seed (8-aligned), 10 int32 -> 64 bytes
-    assert C.sizeof(sr.ReorderParams) == 64
-    assert sr.ReorderParams.seed.offset == 16
+def _c_layout(struct, fields):
+    """sizeof / offsetof of a struct of include/sr.h, compiled with gcc (the header is the
+    authority the ctypes binding must match)."""
+    import subprocess
+    import tempfile
+    body = "".join(f'  printf("%zu\\n", offsetof({struct}, {f}));\n' for f in fields)
+    src = ("#include <stddef.h>\n#include <stdio.h>\n#include \"sr.h\"\n"
+           f"int main(void) {{\n  printf(\"%zu\\n\", sizeof({struct}));\n{body}  return 0;\n}}\n")
+    with tempfile.TemporaryDirectory() as d:
+        c, exe = os.path.join(d, "l.c"), os.path.join(d, "l")
+        with open(c, "w") as f:
+            f.write(src)
+        subprocess.check_call(["gcc", "-I", os.path.join(ROOT, "include"), c, "-o", exe])
+        vals = [int(x) for x in subprocess.check_output([exe]).split()]
+    return vals[0], dict(zip(fields, vals[1:]))
+
+
+@pytest.mark.parametrize("struct,cls", [("sr_reorder_params", "ReorderParams"), ("sr_plan_stats", "PlanStats"),
+                                        ("sr_traffic_model", "TrafficModel")])
+def test_struct_layouts_match_header(sr, struct, cls):
+    T = getattr(sr, cls)
+    fields = [f for f, _ in T._fields_]
+    size, off = _c_layout(struct, fields)
+    assert C.sizeof(T) == size
+    for f in fields:
+        assert getattr(T, f).offset == off[f], f
+
+
+def test_default_params(sr):
     p = sr.default_params()
     assert (p.siglen, p.bsize, p.threshold_size, p.max_bucket, p.seed) == (128, 2, 256, 32, 4)
     assert (p.panel_rows, p.dense_min, p.tile_cols, p.mode) == (64, 2, 64, sr.AUTO)
     assert (p.skip_dense_num, p.skip_dense_den, p.skip_sim_num, p.skip_sim_den) == (1, 10, 1, 10)
+    assert (p.world, p.rank, p.auto_dense_min, p.reserved0) == (1, 0, 0, 0)
 
 
 def test_create_validates_before_touching_a_device(sr):

@@ -107,6 +107,25 @@ def test_worked_example_plan(env, oracle):
     assert M.stats()["dense0"] == 2
 
 
+@pytest.mark.parametrize("case", ["fig1a", "tiny_auto2", "tiny_auto4"])
+def test_auto_decision_threshold_plan(env, oracle, case):
+    """R28: AUTO's DenseRatio0 under auto_dense_min while the plan tiles with dense_min;
+    the library's decision, stats and plan equal the oracle's."""
+    sr, _ = env
+    if case == "fig1a":
+        A, kw = g.fig1a(), dict(_plan_kw(3, 0, 0), dense_min=3, auto_dense_min=2)
+    else:
+        A = g.tiny()
+        kw = dict(_plan_kw(16, 0, 0), dense_min=8, auto_dense_min=2 if case == "tiny_auto2" else 4)
+    ref = oracle.plan(A, **kw)
+    M = sr.SparseMatrix.from_csr(A)
+    M.reorder(sr.default_params(**kw, tile_cols=16))
+    _assert_plan_equal(M, ref)
+    assert M.get_params().auto_dense_min == kw["auto_dense_min"]
+    if case == "fig1a":
+        assert (M.stats()["dense0"], M.stats()["round1"]) == (2, 0)
+
+
 # ------------------------------------------------------------------ numerics over the plan
 @pytest.mark.parametrize("K", [1, 3, 4, 8, 32, 36, 64, 128, 132, 256])
 def test_k_sweep_forced_plan(env, oracle, K):

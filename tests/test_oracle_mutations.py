@@ -31,6 +31,10 @@ MUTATIONS = [
      "if (mode == 0) round1 = !((unsigned __int128)dense0 * d1 > (unsigned __int128)n1 * nnz);",
      "if (mode == 0) round1 = ((unsigned __int128)dense0 * d1 > (unsigned __int128)n1 * nnz);",
      "test_auto_skips_round1_on_clustered_matrix"),
+    ("auto_threshold_ignored",  # R28: the decision's own dense criterion
+     "const int32_t dense_min0 = auto_dense_min > 0 ? auto_dense_min : dense_min;",
+     "const int32_t dense_min0 = dense_min;",
+     "test_auto_decision_threshold_separate_from_execution_threshold"),
     ("sddmm_bound_scale_x100",  # tolerance scale of every GPU SDDMM check
      "if (out_abs) out_abs[j] = accabs * std::abs((double)vals[j]);",
      "if (out_abs) out_abs[j] = 100.0 * accabs * std::abs((double)vals[j]);",

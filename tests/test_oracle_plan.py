@@ -276,6 +276,21 @@ def test_auto_round2_threshold_is_strict(oracle, pairs, expect_round2):
     assert st["round2"] == expect_round2
 
 
+def test_auto_decision_threshold_separate_from_execution_threshold(oracle):
+    """R28: DenseRatio0 of the AUTO decision is taken with the decision's dense
+    criterion auto_dense_min, the tiling the kernels run with uses dense_min.  Fig 1a with
+    execution threshold 3 (no column of a 3-row panel has 3 nnz): decided at 2, DenseRatio0
+    = 2/13 > 1/10 -> round 1 skipped, and the identity plan has no dense nnz; decided at the
+    execution threshold (auto_dense_min 0), DenseRatio0 = 0 -> round 1 runs (hand-derived)."""
+    A = g.fig1a()
+    p = oracle.plan(A, panel_rows=3, dense_min=3, auto_dense_min=2, mode=oracle.MODE_AUTO)
+    st = p["stats"]
+    assert (st["dense0"], st["round1"], st["dense1"]) == (2, 0, 0)
+    assert p["perm1"].tolist() == list(range(6)) and p["dense_ptr"].tolist() == [0, 0, 0]
+    q = oracle.plan(A, panel_rows=3, dense_min=3, auto_dense_min=0, mode=oracle.MODE_AUTO)
+    assert (q["stats"]["dense0"], q["stats"]["round1"]) == (0, 1)
+
+
 def test_plan_modes_consistent(oracle):
     A = g.random_csr(200, 150, 0.04, 9, empty_frac=0.15)
     off = oracle.plan(A, panel_rows=8, mode=oracle.MODE_OFF)
