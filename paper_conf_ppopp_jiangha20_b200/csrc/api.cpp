@@ -183,13 +183,14 @@ int build_identity_plan(sr_csr_s* h, cudaStream_t s) {
     ent[e].x = A.col[e];
     ent[e].y = *reinterpret_cast<const int32_t*>(&A.val[e]);
   }
-  if (A.identity_pos) {
-    std::vector<int32_t> o((size_t)nnz);
+  std::vector<int32_t> o((size_t)nnz);
+  if (A.identity_pos)
     std::iota(o.begin(), o.end(), 0);
-    SR_TRY(P.s_oidx.upload(o, s));
-  } else {
-    SR_TRY(P.s_oidx.upload(A.opos, s));
-  }
+  else
+    std::copy(A.opos.begin(), A.opos.end(), o.begin());
+  ent.resize((size_t)nnz + kEntPad, make_int2(0, 0));
+  o.resize((size_t)nnz + kEntPad, -1);
+  SR_TRY(P.s_oidx.upload(o, s));
   ItemBuilder ib;
   std::vector<int32_t> zero_rows;
   for (int64_t r = 0; r < A.M; ++r) {
@@ -265,13 +266,10 @@ int build_exec_plan(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s) {
   deo.reserve((size_t)T.n_dense() + T.n_dense() / 4);
   int64_t maxd = 0, n_dslots = 0;
   std::vector<int64_t> cur((size_t)PR), stop((size_t)PR);
-  std::vector<int32_t> dcol;
-  dcol.reserve(de.capacity());
   auto pad4 = [&]() {
     while (de.size() % 4) {
       de.push_back(make_int2(0, 0));
       deo.push_back(-1);
-      dcol.push_back(0);
     }
   };
   for (int64_t p = pb; p < pe; ++p) {
@@ -308,7 +306,6 @@ int build_exec_plan(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s) {
               x.x = T.d_slot[e] - (int32_t)(t * TW);
               x.y = *reinterpret_cast<const int32_t*>(&A.val[T.d_cidx[e]]);
               de.push_back(x);
-              dcol.push_back(T.dense_cols[dc0 + T.d_slot[e]]);
               deo.push_back(d_out[e]);
               ++off;
             }
@@ -370,7 +367,6 @@ int build_exec_plan(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s) {
   SR_TRY(P.trp.upload(trp, s));
   SR_TRY(P.d_ent.upload(de, s));
   SR_TRY(P.d_oidx.upload(deo, s));
-  SR_TRY(P.d_col.upload(dcol, s));
   if (n_dslots > 0) {
     SR_TRY(P.dsplit_info.upload(dsplit, s));
     SR_TRY(P.dsplit_counter.alloc((size_t)n_dslots));
@@ -438,6 +434,8 @@ int build_exec_plan(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s) {
       tm.rmw_rows += d && r;
     }
   }
+  se.resize(se.size() + kEntPad, make_int2(0, 0));
+  so.resize(so.size() + kEntPad, -1);
   SR_TRY(P.s_ent.upload(se, s));
   SR_TRY(P.s_oidx.upload(so, s));
   SR_TRY(upload_items(P, ib, n_nonzero, s));

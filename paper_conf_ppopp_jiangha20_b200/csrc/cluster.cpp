@@ -4,18 +4,27 @@
 //
 // Library design (differs from the oracle's plain heap, same result):
 //  * the initial candidates arrive already sorted in heap order (J desc, then (i, j)
-//    asc; R10) from the GPU, so the initial heap is a read cursor over that array;
-//  * pairs re-inserted by Alg 3 line 28 go to an 8-ary heap; each pop takes the larger of
-//    the cursor head and the heap top under the same total order;
-//  * candidate-pair membership (line 27, R9): the initial candidates by binary search in the
-//    key-sorted pair array (the GPU's dedupe output), re-inserted pairs in an open-addressing
-//    hash set.  SR_DEBUG_CLUSTER=1 prints the phase times.
+//    asc; R10) from the GPU, so the initial heap is a read cursor over that array, walked
+//    with software prefetches of the union-find nodes a few pairs ahead;
+//  * pairs re-inserted by Alg 3 line 28 with J > 0 go to an 8-ary heap; each pop takes the
+//    larger of the cursor head and the heap top under the same total order;
+//  * re-inserted pairs with J = 0 (95 % of them on R-MAT) sort after every J > 0 pair, in (i, j)
+//    order: they are appended to an array and sorted once when the J > 0 pairs run out, then
+//    read as a second cursor beside a small min-heap for J = 0 pairs re-inserted after that;
+//  * the exact J of a re-inserted pair (R8) first tests 192-bit column-hash digests of the two
+//    representing rows: disjoint digests prove inter = 0 without reading the column lists;
+//  * union-find parent, cluster size and the deleted flag share one 8-byte node;
+//  * candidate-pair membership (line 27, R9): one open-addressing hash set of the initial and
+//    re-inserted pairs; above 2^26 candidates the initial ones are looked up by binary search
+//    in the key-sorted pair array (the GPU's dedupe output) instead.
+//  SR_DEBUG_CLUSTER=1 prints the phase times.
 // Readings R3-R12 decide everything the paper leaves open.
 #include <algorithm>
 #include <chrono>
 #include <cstdio>
 #include <cstdlib>
 #include <parallel/algorithm>
+#include <queue>
 #include <cstring>
 #include <numeric>
 #include <vector>
@@ -172,6 +181,27 @@ inline void intersect(const int64_t* rowptr, const int32_t* col, int64_t a, int6
   *uni = (uint32_t)(na + nb - n);
 }
 
+// Per-row digest for exact J = 0 detection without touching the column lists: a 192-bit mask
+// of hashed columns and the row length.  Disjoint masks prove that two rows share no column
+// (inter = 0, uni = |S_i| + |S_j|, exactly); overlapping masks fall back to the merge.  On R-MAT
+// (C2) 95 % of Alg 3's re-inserted pairs have J = 0.
+struct __align__(32) RowDigest {
+  uint64_t m[3];
+  uint32_t len, pad;
+};
+inline void digest_bit(uint32_t c, uint32_t* w, uint32_t* bit) {
+  const uint32_t h = c * 0x9E3779B1u;
+  *w = (h >> 8) % 3;
+  *bit = h >> 26;
+}
+
+// Union-find node: parent and cluster size; bit 31 of the size marks a deleted (frozen) cluster.
+struct Node {
+  int32_t parent;
+  uint32_t sz;
+};
+constexpr uint32_t kDeleted = 1u << 31;
+
 }  // namespace
 
 void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t npairs,
@@ -180,13 +210,13 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
   const bool dbg = getenv("SR_DEBUG_CLUSTER") != nullptr;
   auto now = [] { return std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count(); };
   double t0 = now();
-  // initial candidates in heap order; the membership set is built in parallel (the pairs are
-  // distinct), the heap order is a strict total order (R10) so any sort gives the same array
+  // initial candidates in heap order; the heap order is a strict total order (R10), so any
+  // sort gives the same array
   std::vector<Cand> init((size_t)npairs);
-  // membership (line 27, R9): the initial candidates by binary search in their first row's
-  // segment of the key-sorted pair array (when the caller has it), re-inserted pairs in a hash
-  // set; without the key-sorted array every candidate goes into the hash set
-  const bool by_key = pairs_by_key != nullptr;
+  // membership (line 27, R9): one open-addressing hash set of the initial candidates and the
+  // re-inserted pairs (one cache miss per lookup); above 2^26 candidates the initial ones are
+  // found by binary search in the key-sorted pair array instead (memory), if the caller has it
+  const bool by_key = pairs_by_key != nullptr && npairs > (int64_t(1) << 26);
   PairSet members(by_key ? (size_t)npairs / 4 + 16 : (size_t)npairs + (size_t)npairs / 4);
   std::vector<int64_t> seg(by_key ? (size_t)M + 1 : 0);
   if (by_key) {
@@ -201,6 +231,20 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
     }
     return members.contains(key);
   };
+  const double ta = now();
+  std::vector<RowDigest> dig((size_t)M);
+#pragma omp parallel for schedule(dynamic, 4096)
+  for (int64_t r = 0; r < M; ++r) {
+    RowDigest d{};
+    d.len = (uint32_t)(rowptr[r + 1] - rowptr[r]);
+    for (int64_t e = rowptr[r]; e < rowptr[r + 1]; ++e) {
+      uint32_t w, bit;
+      digest_bit((uint32_t)col[e], &w, &bit);
+      d.m[w] |= 1ull << bit;
+    }
+    dig[r] = d;
+  }
+  const double tb = now();
 #pragma omp parallel for schedule(static)
   for (int64_t e = 0; e < npairs; ++e) {
     Cand c;
@@ -222,62 +266,131 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
   const double t1 = now();
   if (!sorted) __gnu_parallel::sort(init.begin(), init.end(), before);
   const double t2 = now();
-  int64_t n_reinsert = 0;
+  int64_t n_reinsert = 0, n_zero = 0;
 
-  std::vector<int32_t> cid((size_t)M), csz((size_t)M, 1);
-  std::vector<uint8_t> dead((size_t)M, 0);
-  std::iota(cid.begin(), cid.end(), 0);
+  std::vector<Node> nd((size_t)M);
+  for (int64_t x = 0; x < M; ++x) nd[x] = Node{(int32_t)x, 1u};
   auto root = [&](int32_t x) {  // path halving
-    while (x != cid[x]) {
-      cid[x] = cid[cid[x]];
-      x = cid[x];
+    while (x != nd[x].parent) {
+      nd[x].parent = nd[nd[x].parent].parent;
+      x = nd[x].parent;
     }
     return x;
   };
-  DHeap extra;
-  size_t cur = 0;
-  int64_t nclusters = M;
-  while ((cur < init.size() || !extra.empty()) && nclusters > 0) {
-    Cand top;
-    if (cur < init.size() && (extra.empty() || before(init[cur], extra.top()))) {
-      top = init[cur++];
+  // Exact J of the representing rows of a re-inserted pair (R8), with the digest early-out.
+  auto similarity = [&](uint32_t lo, uint32_t hi, Cand* c) {
+    const RowDigest &a = dig[lo], &b = dig[hi];
+    c->i = lo;
+    c->j = hi;
+    if (((a.m[0] & b.m[0]) | (a.m[1] & b.m[1]) | (a.m[2] & b.m[2])) == 0) {
+      c->inter = 0;
+      c->uni = a.len + b.len;
     } else {
-      top = extra.top();
-      extra.pop();
+      intersect(rowptr, col, lo, hi, &c->inter, &c->uni);
     }
-    int32_t i = (int32_t)top.i, j = (int32_t)top.j;
-    if (cid[i] == i && cid[j] == j) {
-      if (dead[i] || dead[j]) continue;
+    if (c->uni == 0) c->uni = 1;
+  };
+  // Priority structure (R10 total order: J desc, then (i, j) asc), in three parts that pop in
+  // exactly that order:
+  //  * J > 0: the initial candidates as a sorted cursor (all have J > 0: an LSH candidate shares
+  //    a band key, hence a column) and an 8-ary heap of re-inserted pairs with J > 0;
+  //  * J = 0 (re-inserted pairs only), which pop after every J > 0 pair in (i, j) order: appended
+  //    to a plain array while J > 0 pairs remain, sorted once, then read as a cursor together with
+  //    a min-heap of the J = 0 pairs re-inserted after that point.
+  DHeap extra;
+  std::vector<uint64_t> zero_keys;
+  std::priority_queue<uint64_t, std::vector<uint64_t>, std::greater<uint64_t>> zero_new;
+  bool zero_phase = false;
+  // initial candidates with J = 0 (never produced by the LSH, whose pairs share a column, but
+  // a caller of sr_host_cluster may pass them) sort to the end of `init` and join the J = 0 part
+  size_t init_pos = (size_t)npairs;
+  while (init_pos > 0 && init[init_pos - 1].inter == 0) --init_pos;
+  size_t cur = 0, zc = 0;
+  int64_t nclusters = M;
+  constexpr size_t PF = 32, PF2 = 12;  // prefetch distances over the initial-candidate cursor
+  while (nclusters > 0) {
+    int32_t i, j;
+    if (!zero_phase) {
+      if (cur < init_pos && (extra.empty() || before(init[cur], extra.top()))) {
+        if (cur + PF < init_pos) {
+          __builtin_prefetch(&nd[init[cur + PF].i]);
+          __builtin_prefetch(&nd[init[cur + PF].j]);
+        }
+        if (cur + PF2 < init_pos) {  // second level: the (likely) roots of a nearer pair
+          __builtin_prefetch(&nd[nd[init[cur + PF2].i].parent]);
+          __builtin_prefetch(&nd[nd[init[cur + PF2].j].parent]);
+        }
+        i = (int32_t)init[cur].i;
+        j = (int32_t)init[cur].j;
+        ++cur;
+      } else if (!extra.empty()) {
+        i = (int32_t)extra.top().i;
+        j = (int32_t)extra.top().j;
+        extra.pop();
+      } else {
+        zero_phase = true;
+        if (dbg) fprintf(stderr, "  J>0 phase %.3f s, %lld clusters left, %zu J=0 pairs\n", now() - t2, (long long)nclusters, zero_keys.size());
+        for (size_t e = init_pos; e < init.size(); ++e) zero_keys.push_back(((uint64_t)init[e].i << 32) | init[e].j);
+        __gnu_parallel::sort(zero_keys.begin(), zero_keys.end());
+        continue;
+      }
+    } else {
+      uint64_t key;
+      if (!extra.empty()) {  // a J > 0 pair re-inserted during the J = 0 phase pops first
+        i = (int32_t)extra.top().i;
+        j = (int32_t)extra.top().j;
+        extra.pop();
+        goto have_pair;
+      }
+      if (zc < zero_keys.size() && (zero_new.empty() || zero_keys[zc] < zero_new.top())) {
+        key = zero_keys[zc++];
+      } else if (!zero_new.empty()) {
+        key = zero_new.top();
+        zero_new.pop();
+      } else {
+        break;  // every structure is empty
+      }
+      i = (int32_t)(key >> 32);
+      j = (int32_t)(key & 0xFFFFFFFFu);
+    }
+  have_pair:
+    if (nd[i].parent == i && nd[j].parent == j) {
+      if ((nd[i].sz | nd[j].sz) & kDeleted) continue;
       // the larger cluster absorbs the smaller; equal sizes: smaller index (R6)
-      const bool i_wins = csz[i] > csz[j] || (csz[i] == csz[j] && i < j);
+      const bool i_wins = nd[i].sz > nd[j].sz || (nd[i].sz == nd[j].sz && i < j);
       const int32_t w = i_wins ? i : j, l = i_wins ? j : i;
-      cid[l] = w;
-      csz[w] += csz[l];  // R4
+      nd[l].parent = w;
+      nd[w].sz += nd[l].sz;  // R4
       --nclusters;
-      if (csz[w] >= threshold_size) {  // R7, R5
-        dead[w] = 1;
+      if (nd[w].sz >= (uint32_t)threshold_size) {  // R7, R5
+        nd[w].sz |= kDeleted;
         --nclusters;
       }
     } else {
       i = root(i);
       j = root(j);
-      if (dead[i] || dead[j] || i == j) continue;
+      if (((nd[i].sz | nd[j].sz) & kDeleted) || i == j) continue;
       const uint32_t lo = (uint32_t)std::min(i, j), hi = (uint32_t)std::max(i, j);
       const uint64_t key = ((uint64_t)lo << 32) | hi;
       if (is_candidate(key)) continue;
       Cand c;
-      c.i = lo;
-      c.j = hi;
-      intersect(rowptr, col, lo, hi, &c.inter, &c.uni);  // representing rows (R8)
-      if (c.uni == 0) c.uni = 1;
-      extra.push(c);
+      similarity(lo, hi, &c);  // representing rows (R8)
       members.insert(key);
       ++n_reinsert;
+      if (c.inter > 0) {
+        extra.push(c);
+      } else {
+        ++n_zero;
+        if (zero_phase)
+          zero_new.push(key);
+        else
+          zero_keys.push_back(key);
+      }
     }
   }
   if (dbg)
-    fprintf(stderr, "cluster_rows: build %.3f s, sort %.3f s (sorted=%d), loop %.3f s, %lld re-inserted\n", t1 - t0,
-            t2 - t1, (int)sorted, now() - t2, (long long)n_reinsert);
+    fprintf(stderr, "cluster_rows: set %.3f s, digests %.3f s, build %.3f s, sort %.3f s (sorted=%d), loop %.3f s, %lld re-inserted (%lld with J = 0)\n",
+            ta - t0, tb - ta, t1 - tb, t2 - t1, (int)sorted, now() - t2, (long long)n_reinsert, (long long)n_zero);
   // rule B (R11): clusters of >= 2 rows by ascending root, then singletons ascending
   std::vector<int32_t> r_of((size_t)M);
   std::vector<int64_t> count((size_t)M + 1, 0);

@@ -842,103 +842,6 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) spmm_
   }
 }
 
-// SpMM dense tiles through L1 instead of shared memory ("L1 staging"): one CTA per unit, its
-// warps walk the unit's tiles without any barrier and gather the dense columns' B rows with
-// L1-allocating 128-bit loads; the first warp to touch a dense column brings its row into
-// L1 and the other rows of the panel hit it there (the reuse ASpT gets from shared memory).
-// Entries carry their global column id (d_col, tile-major like d_ent).
-template <int LPG, int VEC, int U, int RPW>
-__global__ void __launch_bounds__(kDenseWarps * 32, 4) spmm_dense_l1_kernel(
-    const DUnit* __restrict__ units, const VTile* __restrict__ vtiles, const int32_t* __restrict__ trp,
-    const int2* __restrict__ ent, const int32_t* __restrict__ dcol, const int32_t* __restrict__ dense_out,
-    const float* __restrict__ B, int64_t ldb, float* __restrict__ C, int64_t ldc, int K, int TS, int P,
-    float* __restrict__ scratch, const int2* __restrict__ split_info, int* __restrict__ split_counter) {
-  constexpr int G = 32 / LPG;
-  constexpr int KC = LPG * VEC;
-  __shared__ int last_ticket;
-  const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
-  const int warp = threadIdx.x >> 5;
-  const DUnit u = units[blockIdx.x];
-  const int r0 = warp * RPW;
-  const int out_row = (lane < RPW && r0 + lane < u.nrows) ? dense_out[u.q0 + r0 + lane] : -1;
-  for (int k0 = 0; k0 < K; k0 += KC) {
-    const int kk = k0 + lg * VEC;
-    const bool kv = kk < K;
-    Frag<VEC> acc[RPW];
-#pragma unroll
-    for (int i = 0; i < RPW; ++i) acc[i].zero();
-    if (r0 < u.nrows) {
-      for (int t = 0; t < u.nvt; ++t) {
-        const int vt = u.vt0 + t;
-        const int ent0 = __ldg(&vtiles[vt].ent0);
-        const int bnd = lane <= RPW ? __ldg(trp + (int64_t)vt * TS + r0 + lane) : 0;
-        const int e_lo = __shfl_sync(FULL, bnd, 0), e_hi = __shfl_sync(FULL, bnd, RPW);
-        for (int e = e_lo; e < e_hi; e += 32) {
-          const int n = min(32, e_hi - e);
-          const int2 my = lane < n ? __ldcs(ent + ent0 + e + lane) : make_int2(0, 0);
-          const int myc = lane < n ? __ldcs(dcol + ent0 + e + lane) : 0;
-#pragma unroll
-          for (int i = 0; i < RPW; ++i) {
-            const int a = max(0, __shfl_sync(FULL, bnd, i) - e), b = min(n, __shfl_sync(FULL, bnd, i + 1) - e);
-            for (int base = a; base < b; base += G * U) {
-              Frag<VEC> bv[U];
-              float av[U];
-#pragma unroll
-              for (int uu = 0; uu < U; ++uu) {
-                const int j = base + uu * G + g;
-                const int c = __shfl_sync(FULL, myc, j & 31);
-                const float v = __int_as_float(__shfl_sync(FULL, my.y, j & 31));
-                const bool ok = j < b && kv;
-                av[uu] = ok ? v : 0.f;
-                if (ok) bv[uu].load_g(B + (int64_t)c * ldb + kk); else bv[uu].zero();
-              }
-#pragma unroll
-              for (int uu = 0; uu < U; ++uu) acc[i].fma(av[uu], bv[uu]);
-            }
-          }
-        }
-      }
-    }
-#pragma unroll
-    for (int i = 0; i < RPW; ++i) {
-#pragma unroll
-      for (int off = LPG; off < 32; off <<= 1) acc[i].xor_add(off);
-      const int orow = __shfl_sync(FULL, out_row, i);
-      if (r0 + i < u.nrows && g == 0 && kv) {
-        if (u.split >= 0)
-          acc[i].store(scratch + ((int64_t)u.split * P + r0 + i) * K + kk);
-        else if (orow >= 0)
-          acc[i].store_cs(C + (int64_t)orow * ldc + kk);
-      }
-    }
-  }
-  if (u.split >= 0) {
-    __threadfence();
-    __syncthreads();
-    const int2 si = split_info[u.split];
-    if (threadIdx.x == 0) last_ticket = (atomicAdd(split_counter + si.x, 1) == si.y - 1);
-    __syncthreads();
-    if (!last_ticket) return;
-    __threadfence();
-    for (int i = 0; i < RPW; ++i) {
-      const int orow = __shfl_sync(FULL, out_row, i);
-      if (r0 + i >= u.nrows || orow < 0) continue;
-      for (int k = lane * VEC; k < K; k += 32 * VEC) {
-        Frag<VEC> s;
-        s.zero();
-        for (int c = 0; c < si.y; ++c) {
-          Frag<VEC> part;
-          part.load_cg(scratch + ((int64_t)(si.x + c) * P + r0 + i) * K + k);
-          s.add(part);
-        }
-        s.store_cs(C + (int64_t)orow * ldc + k);
-      }
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) split_counter[si.x] = 0;
-  }
-}
-
 // SDDMM dense tiles.  Lane geometry as phase S: LPG lanes × NCH chunks of LPG·VEC columns
 // cover one nnz (K=128: 8 lanes × 4 float4, 4 nnz per warp step, 3-step shuffle reduction).
 // X fragments of the current row come from global memory (L1-resident across the tiles);
@@ -1039,281 +942,6 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) sddmm
   }
 }
 
-// ------------------------------------------------------------------ phase D, cooperative staging
-// One CTA (8 warps) per work unit (<= kMaxUnitTiles virtual tiles of one panel), several
-// CTAs per SM.  All 256 threads stage a tile — its dense columns' B/Y rows (16-byte
-// cp.async = LDGSTS, spread over every lane of the CTA), its panel-row offsets and its entry
-// block — into one of two shared-memory buffers while the previous tile is computed from the
-// other; one CTA barrier per tile.  Latency is hidden by the other resident CTAs and by the
-// double buffer instead of a producer warp and an mbarrier ring, so the staged bytes in
-// flight scale with the number of issuing lanes (the TMA producer of the persistent engine
-// staged at 1.6-2.4 TB/s, profiles/r01/NOTES.md).  The arithmetic is the persistent
-// engine's: per nnz one broadcast LDS.64 of (slot, value), one LDS.128 of the staged row,
-// four FFMA (SDDMM: 8 lanes × 4 float4 per nnz and a 3-step shuffle reduction).
-template <int VEC>
-__device__ __forceinline__ void cp_async_v(void* s, const void* g);
-template <>
-__device__ __forceinline__ void cp_async_v<4>(void* s, const void* g) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(s)), "l"(g) : "memory");
-}
-template <>
-__device__ __forceinline__ void cp_async_v<1>(void* s, const void* g) {
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(s)), "l"(g) : "memory");
-}
-__device__ __forceinline__ void cp_async16(void* s, const void* g) { cp_async_v<4>(s, g); }
-__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_wait() {
-  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
-}
-
-constexpr int kD2Threads = 256;
-
-// stage = [staged rows: kMaxExecTile × KCP floats][trp: TS ints][entries][SDDMM output indices]
-struct D2Layout {
-  int KCP, TS;
-  bool oidx;
-  __host__ __device__ size_t trp_off() const { return (size_t)kMaxExecTile * KCP * 4; }
-  __host__ __device__ size_t ent_off() const { return (trp_off() + (size_t)TS * 4 + 15) / 16 * 16; }
-  __host__ __device__ size_t oidx_off() const { return ent_off() + (size_t)kMaxTileEntries * 8; }
-  __host__ __device__ size_t bytes() const {
-    return (oidx_off() + (oidx ? (size_t)kMaxTileEntries * 4 : 0) + 127) / 128 * 128;
-  }
-};
-
-template <int VEC>
-__device__ __forceinline__ void d2_stage(char* st, const D2Layout& L, const VTile& v, int vt,
-                                         const int32_t* __restrict__ dense_cols, const int32_t* __restrict__ trp,
-                                         const int2* __restrict__ ent, const int32_t* __restrict__ oidx,
-                                         const float* __restrict__ src, int64_t ld, int k0, int kw) {
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  float* bs = reinterpret_cast<float*>(st);
-  const int cpr = kw / VEC;  // chunks per staged row (VEC divides kw on the vector path)
-  // warp w stages rows w, w+8, ... (<= 8 rows of a <= 64-column tile): one load of their
-  // column ids (lanes 0..7), then per row a shuffle and the row's chunks over the lanes
-  const int myc = lane < 8 && warp + 8 * lane < v.ncols ? __ldg(dense_cols + v.col0 + warp + 8 * lane) : 0;
-  const float* s0 = src + k0;
-#pragma unroll
-  for (int m = 0; m < kMaxExecTile / 8; ++m) {
-    const int j = warp + 8 * m;
-    const int col = __shfl_sync(FULL, myc, m);
-    if (j < v.ncols) {
-      const float* row = s0 + (int64_t)col * ld;
-      float* dst = bs + (size_t)j * L.KCP;
-      for (int q = lane; q < cpr; q += 32) cp_async_v<VEC>(dst + q * VEC, row + q * VEC);
-    }
-  }
-  if (tid < L.TS / 4) cp_async16(st + L.trp_off() + tid * 16, trp + (int64_t)vt * L.TS + tid * 4);
-  if (tid < v.nent / 2) cp_async16(st + L.ent_off() + tid * 16, ent + v.ent0 + tid * 2);
-  if (L.oidx && tid < v.nent / 4) cp_async16(st + L.oidx_off() + tid * 16, oidx + v.ent0 + tid * 4);
-}
-
-template <int LPG, int VEC, int U, int RPW>
-__global__ void __launch_bounds__(kD2Threads, 3) spmm_dense2_kernel(
-    const DUnit* __restrict__ units, const VTile* __restrict__ vtiles, const int32_t* __restrict__ dense_cols,
-    const int32_t* __restrict__ trp, const int2* __restrict__ ent, const int32_t* __restrict__ dense_out,
-    const float* __restrict__ B, int64_t ldb, float* __restrict__ C, int64_t ldc, int K, int TS, int P,
-    float* __restrict__ scratch, const int2* __restrict__ split_info, int* __restrict__ split_counter) {
-  constexpr int G = 32 / LPG;
-  constexpr int KC = LPG * VEC;
-  extern __shared__ __align__(128) char smem_raw[];
-  __shared__ int last_ticket;
-  const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
-  const int warp = threadIdx.x >> 5;
-  const D2Layout L{((KC + 3) & ~3), TS, false};
-  const size_t SB = L.bytes();
-  const DUnit u = units[blockIdx.x];
-  const int r0 = warp * RPW;
-  const int out_row = (lane < RPW && r0 + lane < u.nrows) ? dense_out[u.q0 + r0 + lane] : -1;
-  for (int k0 = 0; k0 < K; k0 += KC) {
-    const int kw = min(KC, K - k0);
-    const int kk = k0 + lg * VEC;
-    const bool kv = kk < K;
-    Frag<VEC> acc[RPW];
-#pragma unroll
-    for (int i = 0; i < RPW; ++i) acc[i].zero();
-    d2_stage<VEC>(smem_raw, L, vtiles[u.vt0], u.vt0, dense_cols, trp, ent, nullptr, B, ldb, k0, kw);
-    cp_commit();
-    for (int t = 0; t < u.nvt; ++t) {
-      if (t + 1 < u.nvt)
-        d2_stage<VEC>(smem_raw + ((t + 1) & 1) * SB, L, vtiles[u.vt0 + t + 1], u.vt0 + t + 1, dense_cols, trp, ent,
-                      nullptr, B, ldb, k0, kw);
-      cp_commit();
-      cp_wait<1>();     // this thread's copies of tile t have landed
-      __syncthreads();  // ... and everyone else's
-      const char* base = smem_raw + (t & 1) * SB;
-      if (r0 < u.nrows && lg * VEC < kw) {
-        const float* tcol = reinterpret_cast<const float*>(base) + lg * VEC;
-        const int32_t* rp = reinterpret_cast<const int32_t*>(base + L.trp_off()) + r0;
-        const int2* es = reinterpret_cast<const int2*>(base + L.ent_off());
-#pragma unroll
-        for (int i = 0; i < RPW; ++i) {
-          const int b0 = rp[i], b1 = rp[i + 1];
-          int e = b0 + g;
-          for (; e + (U - 1) * G < b1; e += U * G) {
-            int2 en[U];
-#pragma unroll
-            for (int uu = 0; uu < U; ++uu) en[uu] = es[e + uu * G];
-            Frag<VEC> bv[U];
-#pragma unroll
-            for (int uu = 0; uu < U; ++uu) bv[uu].load_s(tcol + (size_t)en[uu].x * L.KCP);
-#pragma unroll
-            for (int uu = 0; uu < U; ++uu) acc[i].fma(__int_as_float(en[uu].y), bv[uu]);
-          }
-          for (; e < b1; e += G) {
-            const int2 en = es[e];
-            Frag<VEC> bv;
-            bv.load_s(tcol + (size_t)en.x * L.KCP);
-            acc[i].fma(__int_as_float(en.y), bv);
-          }
-        }
-      }
-      __syncthreads();  // buffer (t & 1) may be restaged by the next iteration
-    }
-#pragma unroll
-    for (int i = 0; i < RPW; ++i) {
-#pragma unroll
-      for (int off = LPG; off < 32; off <<= 1) acc[i].xor_add(off);
-      const int orow = __shfl_sync(FULL, out_row, i);
-      if (r0 + i < u.nrows && g == 0 && kv) {
-        if (u.split >= 0)
-          acc[i].store(scratch + ((int64_t)u.split * P + r0 + i) * K + kk);
-        else if (orow >= 0)
-          acc[i].store_cs(C + (int64_t)orow * ldc + kk);
-      }
-    }
-  }
-  if (u.split >= 0) {
-    // giant panel split over several units: the last unit to finish sums the chunk partials in
-    // unit order (deterministic) and writes the panel's dense rows
-    __threadfence();
-    __syncthreads();
-    const int2 si = split_info[u.split];
-    if (threadIdx.x == 0) last_ticket = (atomicAdd(split_counter + si.x, 1) == si.y - 1);
-    __syncthreads();
-    if (!last_ticket) return;
-    __threadfence();
-    const int kq = (K + VEC - 1) / VEC;
-    const int64_t cstride = (int64_t)P * K;
-    for (int item = threadIdx.x; item < u.nrows * kq; item += kD2Threads) {
-      const int r = item / kq, k = (item - r * kq) * VEC;
-      const int orow = dense_out[u.q0 + r];
-      if (orow < 0) continue;
-      const float* src = scratch + ((int64_t)si.x * P + r) * K + k;
-      Frag<VEC> sacc;
-      sacc.zero();
-      int c = 0;
-      for (; c + 4 <= si.y; c += 4) {
-        Frag<VEC> p0, p1, p2, p3;
-        p0.load_cg(src + (c + 0) * cstride);
-        p1.load_cg(src + (c + 1) * cstride);
-        p2.load_cg(src + (c + 2) * cstride);
-        p3.load_cg(src + (c + 3) * cstride);
-        sacc.add(p0); sacc.add(p1); sacc.add(p2); sacc.add(p3);
-      }
-      for (; c < si.y; ++c) {
-        Frag<VEC> p0;
-        p0.load_cg(src + c * cstride);
-        sacc.add(p0);
-      }
-      sacc.store_cs(C + (int64_t)orow * ldc + k);
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) split_counter[si.x] = 0;
-  }
-}
-
-template <int LPG, int VEC, int U, int NCH, int RPW>
-__global__ void __launch_bounds__(kD2Threads, 3) sddmm_dense2_kernel(
-    const DUnit* __restrict__ units, const VTile* __restrict__ vtiles, const int32_t* __restrict__ dense_cols,
-    const int32_t* __restrict__ trp, const int2* __restrict__ ent, const int32_t* __restrict__ d_oidx,
-    const int32_t* __restrict__ pos_xrow, const float* __restrict__ X, int64_t ldx, const float* __restrict__ Y,
-    int64_t ldy, int K, int TS, float* __restrict__ out) {
-  constexpr int G = 32 / LPG;
-  constexpr int KC = LPG * VEC;   // columns of one chunk
-  constexpr int KCP = NCH * KC;   // columns staged per pass (slot stride)
-  extern __shared__ __align__(128) char smem_raw[];
-  const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
-  const int warp = threadIdx.x >> 5;
-  const D2Layout L{KCP, TS, true};
-  const size_t SB = L.bytes();
-  const DUnit u = units[blockIdx.x];
-  const int r0 = warp * RPW;
-  const int xrow = (lane < RPW && r0 + lane < u.nrows) ? pos_xrow[u.q0 + r0 + lane] : 0;
-  for (int k0 = 0; k0 < K; k0 += KCP) {
-    const int kw = min(KCP, K - k0);
-    d2_stage<VEC>(smem_raw, L, vtiles[u.vt0], u.vt0, dense_cols, trp, ent, d_oidx, Y, ldy, k0, kw);
-    cp_commit();
-    for (int t = 0; t < u.nvt; ++t) {
-      if (t + 1 < u.nvt)
-        d2_stage<VEC>(smem_raw + ((t + 1) & 1) * SB, L, vtiles[u.vt0 + t + 1], u.vt0 + t + 1, dense_cols, trp, ent,
-                      d_oidx, Y, ldy, k0, kw);
-      cp_commit();
-      cp_wait<1>();
-      __syncthreads();
-      const char* base = smem_raw + (t & 1) * SB;
-      if (r0 < u.nrows) {
-        const float* tile = reinterpret_cast<const float*>(base);
-        const int32_t* rp = reinterpret_cast<const int32_t*>(base + L.trp_off());
-        const int2* es = reinterpret_cast<const int2*>(base + L.ent_off());
-        const int32_t* os = reinterpret_cast<const int32_t*>(base + L.oidx_off());
-#pragma unroll 1
-        for (int i = 0; i < RPW; ++i) {
-          const int b0 = rp[r0 + i], b1 = rp[r0 + i + 1];
-          const int xr_i = __shfl_sync(FULL, xrow, i);
-          if (b0 >= b1) continue;
-          Frag<VEC> x[NCH];
-          const float* xr = X + (int64_t)xr_i * ldx + k0;
-#pragma unroll
-          for (int c = 0; c < NCH; ++c) {
-            if (c * KC + lg * VEC < kw) x[c].load_g(xr + c * KC + lg * VEC); else x[c].zero();
-          }
-          for (int bse = b0; bse < b1; bse += G * U) {
-            float part[U];
-            int2 en[U];
-#pragma unroll
-            for (int uu = 0; uu < U; ++uu) {
-              const int j = bse + uu * G + g;
-              en[uu] = j < b1 ? es[j] : make_int2(0, 0);
-            }
-#pragma unroll
-            for (int uu = 0; uu < U; ++uu) {
-              float d = 0.f;
-#pragma unroll
-              for (int c = 0; c < NCH; ++c) {
-                if (c * KC + lg * VEC < kw) {
-                  Frag<VEC> y;
-                  y.load_s(tile + (size_t)en[uu].x * KCP + c * KC + lg * VEC);
-                  d += x[c].dot(y);
-                }
-              }
-              part[uu] = d;
-            }
-#pragma unroll
-            for (int uu = 0; uu < U; ++uu) {
-#pragma unroll
-              for (int off = LPG / 2; off > 0; off >>= 1) part[uu] += __shfl_xor_sync(FULL, part[uu], off);
-            }
-            if (lg == 0) {
-#pragma unroll
-              for (int uu = 0; uu < U; ++uu) {
-                const int j = bse + uu * G + g;
-                if (j < b1) {
-                  const int o = os[j];
-                  float res = __int_as_float(en[uu].y) * part[uu];
-                  if (k0 > 0) res += out[o];
-                  out[o] = res;
-                }
-              }
-            }
-          }
-        }
-      }
-      __syncthreads();
-    }
-  }
-}
-
 // ------------------------------------------------------------------ host dispatch
 inline int next_pow2(int x) {
   int p = 1;
@@ -1364,31 +992,15 @@ bool make_row_gather_map(CUtensorMap* map, const float* base, int64_t rows, int6
                 CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-// Phase-D engine (SR_DENSE_ENGINE): "tma" = persistent producer/consumer engine (default),
-// "coop" = one CTA per unit with cooperative cp.async staging, "l1" = L1 staging (SpMM only).
-// Measured trade-off in profiles/r01/NOTES.md: coop wins at low dense thresholds (C2 dense_min
-// 2, C4 dense_min 4), tma on the hub-panel-dominated C2 default and on C5.
-int dense_engine() {  // 0 = coop, 1 = l1, 2 = tma
-  static const int v = [] {
-    const char* d = getenv("SR_DENSE_ENGINE");
-    if (d && std::string(d) == "l1") return 1;
-    if (d && std::string(d) == "coop") return 0;
-    return 2;
-  }();
-  return v;
+// Phase-S kernel choice (measurement knob SR_PHASE_S; profiles/r01/NOTES.md, profiles/r02/NOTES.md):
+// 1 (default) = row-group task kernels where K allows them, 0 = one-row-per-warp kernels (also
+// the path for K that is not a multiple of 32).
+int env_int(const char* name, int dflt) {
+  const char* d = getenv(name);
+  return d ? atoi(d) : dflt;
 }
-
-// Phase-S kernel choice (SR_SPARSE_VARIANT, measurement knob; profiles/r01/NOTES.md):
-// default (7) = row-group task kernels: SpMM K = 128·p float4 lanes U 4 at 8 CTAs/SM, SpMM
-// K = 32·p float lanes U 8 at 8 CTAs/SM, SDDMM K = 32·NCH <= 128 8-lane groups U 2 at 4 CTAs/SM
-// with the permuted entry layout (4 = lane-order layout);
-// 0 = one-row-per-warp kernels (U 2 / 8 CTAs); 1, 3 = row kernels at other occupancy points;
-// 4-6 = task kernels at other (U, CTAs/SM) points.
-int sparse_variant() {
-  static const int v = [] {
-    const char* d = getenv("SR_SPARSE_VARIANT");
-    return d ? atoi(d) : 7;
-  }();
+bool task_kernels() {
+  static const bool v = env_int("SR_PHASE_S", 1) != 0;
   return v;
 }
 
@@ -1432,29 +1044,7 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
       return SR_OK;
     };
     if (P.profiling) SR_TRY(prof_begin(P, 1, s));
-    if (dense_engine() == 0) {
-      const size_t smem2 = 2 * D2Layout{((KC + 3) & ~3), P.trp_stride, false}.bytes();
-      auto d2 = [&](auto kern) -> int {
-        SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem2));
-        kern<<<(unsigned)P.n_units, kD2Threads, smem2, s>>>(
-            P.units.p, P.vtiles.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.dense_out.p, B, ldb, C, ldc, (int)K,
-            P.trp_stride, P.panel_rows, P.dscratch.p, P.dsplit_info.p, P.dsplit_counter.p);
-        SR_CUDA_TRY(cudaGetLastError());
-        return SR_OK;
-      };
-      if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(d2(spmm_dense2_kernel<LPG, VEC, UD, 8>));
-      else SR_TRY(d2(spmm_dense2_kernel<LPG, VEC, UD, 16>));
-    } else if (dense_engine() == 1) {  // L1 staging (SR_DENSE_ENGINE=l1)
-      auto l1 = [&](auto kern) -> int {
-        kern<<<(unsigned)P.n_units, kDenseWarps * 32, 0, s>>>(
-            P.units.p, P.vtiles.p, P.trp.p, P.d_ent.p, P.d_col.p, P.dense_out.p, B, ldb, C, ldc, (int)K,
-            P.trp_stride, P.panel_rows, P.dscratch.p, P.dsplit_info.p, P.dsplit_counter.p);
-        SR_CUDA_TRY(cudaGetLastError());
-        return SR_OK;
-      };
-      if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(l1(spmm_dense_l1_kernel<LPG, VEC, 2, 8>));
-      else SR_TRY(l1(spmm_dense_l1_kernel<LPG, VEC, 2, 16>));
-    } else if (P.panel_rows <= 8 * kDenseWarps) {
+    if (P.panel_rows <= 8 * kDenseWarps) {
       SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 8>));
     } else {
       SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 16>));
@@ -1469,10 +1059,9 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
     }
     const unsigned grid = (unsigned)((P.n_items + kSparseWarps - 1) / kSparseWarps);
     if (P.profiling) SR_TRY(prof_begin(P, 2, s));
-    const int var = sparse_variant();
     // row-group task kernels: K = 128·passes (float4 lanes) or 32·passes (float lanes)
     const int tvec = (VEC == 4 && K % 128 == 0) ? 4 : (K % 32 == 0 ? 1 : 0);
-    if (tvec && ldb * 4 < (1ll << 32) && var >= 4 && var <= 10 && P.n_tasks > 0) {
+    if (tvec && ldb * 4 < (1ll << 32) && task_kernels() && P.n_tasks > 0) {
       const unsigned tgrid = (unsigned)((P.n_tasks + kSparseWarps - 1) / kSparseWarps);
       const int pass = 32 * tvec;
       auto tk = [&](auto kern) {
@@ -1481,19 +1070,10 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
                                                     B + k0, (uint32_t)(ldb * 4), C + k0, ldc, (int)K, k0, P.scratch.p,
                                                     P.split_info.p, P.split_counter.p);
       };
-      if (tvec == 4) {
-        switch (var) {
-          case 4: tk(spmm_task_kernel<4, 6, 4>); break;
-          case 5: tk(spmm_task_kernel<8, 4, 4>); break;
-          case 6: tk(spmm_task_kernel<2, 8, 4>); break;
-          default: tk(spmm_task_kernel<4, 8, 4>); break;
-        }
-      } else {
-        switch (var) {
-          case 5: tk(spmm_task_kernel<16, 4, 1>); break;
-          default: tk(spmm_task_kernel<8, 8, 1>); break;
-        }
-      }
+      if (tvec == 4)
+        tk(spmm_task_kernel<4, 8, 4>);  // U 4 gathers per lane, 8 CTAs (64 warps) per SM
+      else
+        tk(spmm_task_kernel<8, 8, 1>);
       SR_CUDA_TRY(cudaGetLastError());
       if (P.profiling) SR_TRY(prof_end(P, s));
       ++*launches;
@@ -1503,14 +1083,8 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
       kern<<<grid, kSparseWarps * 32, 0, s>>>(P.items.p, P.item_meta.p, P.n_items, P.s_ent.p, B, ldb, C, ldc, (int)K,
                                                P.scratch.p, P.split_info.p, P.split_counter.p);
     };
-    // occupancy beats per-warp memory parallelism here (profiles/r01): U=2 gathers per lane
-    // at 8 CTAs (64 warps) per SM.  SR_SPARSE_VARIANT (tuning knob): 1 = U 4 / 6 CTAs,
-    // 3 = U 8 / 4 CTAs.
-    switch (sparse_variant()) {
-      case 1: go(spmm_sparse_kernel<LPG, VEC, (U > 4 ? 4 : U), 6>); break;
-      case 3: go(spmm_sparse_kernel<LPG, VEC, U, 4>); break;
-      default: go(spmm_sparse_kernel<LPG, VEC, 2, 8>); break;
-    }
+    // one row (or chunk) per warp: U=2 gathers per lane at 8 CTAs (64 warps) per SM (profiles/r01)
+    go(spmm_sparse_kernel<LPG, VEC, 2, 8>);
     SR_CUDA_TRY(cudaGetLastError());
     if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;
@@ -1543,19 +1117,7 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
     };
     constexpr int UD = 4;
     if (P.profiling) SR_TRY(prof_begin(P, 3, s));
-    if (dense_engine() != 2) {
-      const size_t smem2 = 2 * D2Layout{NCH_D * KC, P.trp_stride, true}.bytes();
-      auto d2 = [&](auto kern) -> int {
-        SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem2));
-        kern<<<(unsigned)P.n_units, kD2Threads, smem2, s>>>(P.units.p, P.vtiles.p, P.dense_cols.p, P.trp.p, P.d_ent.p,
-                                                           P.d_oidx.p, P.pos_xrow.p, X, ldx, Y, ldy, (int)K,
-                                                           P.trp_stride, out);
-        SR_CUDA_TRY(cudaGetLastError());
-        return SR_OK;
-      };
-      if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(d2(sddmm_dense2_kernel<LPG, VEC, 2, NCH_D, 8>));
-      else SR_TRY(d2(sddmm_dense2_kernel<LPG, VEC, 2, NCH_D, 16>));
-    } else if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 8>));
+    if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 8>));
     else SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 16>));
     if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;
@@ -1563,20 +1125,15 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
   if (P.n_sitems > 0) {
     const unsigned grid = (unsigned)((P.n_sitems + kSparseWarps - 1) / kSparseWarps);
     if (P.profiling) SR_TRY(prof_begin(P, 4, s));
-    const int var = sparse_variant();
-    if (LPG == 8 && VEC == 4 && NCH <= 4 && K == 32 * NCH && ldy * 4 < (1ll << 32) && var >= 4 && var <= 10 &&
+    if (LPG == 8 && VEC == 4 && NCH <= 4 && K == 32 * NCH && ldy * 4 < (1ll << 32) && task_kernels() &&
         P.n_stasks > 0) {
       const unsigned tgrid = (unsigned)((P.n_stasks + kSparseWarps - 1) / kSparseWarps);
       auto tk = [&](auto kern) {
-        kern<<<tgrid, kSparseWarps * 32, 0, s>>>(P.stasks.p, P.n_stasks, P.items.p, P.s_ent.p, P.s_oidx.p, X, ldx,
-                                                  Y, (uint32_t)(ldy * 4), out);
+        kern<<<tgrid, kSparseWarps * 32, 0, s>>>(P.stasks.p, P.n_stasks, P.items.p, P.s_ent.p, P.s_oidx.p, X,
+                                                  ldx, Y, (uint32_t)(ldy * 4), out);
       };
       constexpr int NC = NCH > 4 ? 4 : NCH;  // (NCH <= 4 guarded above; keeps NCH 8 instantiable)
-      switch (var) {
-        case 4: tk(sddmm_task_kernel<NC, 2, 4>); break;  // entries in lane order (shuffled values)
-        case 5: tk(sddmm_task_kernel<NC, 1, 6, true>); break;
-        default: tk(sddmm_task_kernel<NC, 2, 4, true>); break;
-      }
+      tk(sddmm_task_kernel<NC, 2, 4, true>);
       SR_CUDA_TRY(cudaGetLastError());
       if (P.profiling) SR_TRY(prof_end(P, s));
       ++*launches;
@@ -1586,12 +1143,7 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
       kern<<<grid, kSparseWarps * 32, 0, s>>>(P.items.p, P.n_sitems, P.s_ent.p, P.s_oidx.p, X, ldx, Y, ldy, (int)K,
                                                out);
     };
-    // SR_SPARSE_VARIANT (tuning knob) also selects the SDDMM occupancy point
-    switch (sparse_variant()) {
-      case 1: go(sddmm_sparse_kernel<LPG, VEC, U, NCH, 1>); break;
-      case 2: go(sddmm_sparse_kernel<LPG, VEC, 1, NCH, 6>); break;
-      default: go(sddmm_sparse_kernel<LPG, VEC, U, NCH, 4>); break;
-    }
+    go(sddmm_sparse_kernel<LPG, VEC, U, NCH, 4>);
     SR_CUDA_TRY(cudaGetLastError());
     if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;

@@ -100,6 +100,10 @@ struct __align__(16) Item {
   int32_t out;   // SpMM output row (original id, or packed shard index)
 };
 
+// The phase-S entry streams carry kEntPad trailing padding entries ({0, 0}, output index -1) so
+// a kernel may load entries in pairs past the end of its last task.
+constexpr int kEntPad = 8;
+
 constexpr uint32_t kItemRMW = 1u << 31;    // C[out] += partial (row also has dense-tile nnz)
 constexpr uint32_t kItemSplit = 1u << 30;  // partial of a split long row -> scratch slot
 constexpr uint32_t kItemSlotMask = (1u << 30) - 1;
@@ -139,7 +143,6 @@ struct DevPlan {
   DevBuf<int32_t> drow_ptr;   // positions -> dense nnz offsets (only "row has dense nnz" is used)
   DevBuf<int2> d_ent;         // tile-major {slot in tile, __float_as_int(val)}
   DevBuf<int32_t> d_oidx;     // SDDMM output index per dense nnz (tile-major)
-  DevBuf<int32_t> d_col;      // global column id per dense nnz (tile-major; L1-staging kernel)
   DevBuf<int2> dsplit_info;   // per split unit: {first slot, nchunks}
   DevBuf<int32_t> dsplit_counter;
   int64_t n_dslots = 0;

@@ -1,8 +1,10 @@
 """Row-panel sharding across GPUs (north_star).
 
-One process per GPU (torchrun).  Every rank builds the same plan (the reorder is
-deterministic per seed) and keeps its nnz-balanced contiguous panel range
-(`sr_reorder(world, rank)`); B/X/Y are replicated.  The step needs no collective.  When the
+One process per GPU (torchrun).  The plan is built once: rank 0 reorders the whole matrix
+(`sr_reorder`), broadcasts the plan image (`broadcast_bytes`), and every rank installs its
+nnz-balanced contiguous panel range with `sr_plan_load(world, rank)` (`load_shard`; the
+reorder is deterministic per seed, so `sr_reorder(world, rank)` on every rank gives the same
+shards at the cost of repeating it).  B/X/Y are replicated.  The step needs no collective.  When the
 caller wants the full C (or the full SDDMM values) on every rank, `gather_spmm` /
 `gather_sddmm` all-gather the packed shard outputs (NCCL over NVLink via
 torch.distributed, padded to the largest shard) and scatter them back to original
@@ -14,6 +16,28 @@ import torch
 import torch.distributed as tdist
 
 import paper_conf_ppopp_jiangha20_b200 as sr
+
+
+def broadcast_bytes(data: bytes | None, src: int = 0, group=None, device=None) -> bytes:
+    """Broadcast a byte string from rank `src` (the plan image): its length, then the bytes as a
+    uint8 tensor (on `device`: a CUDA device for NCCL, None = CPU for gloo)."""
+    rank = tdist.get_rank(group)
+    n = torch.tensor([len(data) if rank == src else 0], dtype=torch.int64, device=device)
+    tdist.broadcast(n, src, group=group)
+    if rank == src:
+        buf = torch.frombuffer(bytearray(data), dtype=torch.uint8).to(device) if n.item() else \
+            torch.empty(0, dtype=torch.uint8, device=device)
+    else:
+        buf = torch.empty(int(n.item()), dtype=torch.uint8, device=device)
+    tdist.broadcast(buf, src, group=group)
+    return bytes(buf.cpu().numpy().tobytes())
+
+
+def load_shard(A, image: bytes, world: int, rank: int, device: int) -> "sr.SparseMatrix":
+    """A handle of matrix A on `device` holding shard `rank` of `world` of a saved plan."""
+    M = sr.SparseMatrix.from_csr(A, device=device)
+    M.load_plan(image, world=world, rank=rank)
+    return M
 
 
 def allgather_padded(t: torch.Tensor, group=None) -> list:

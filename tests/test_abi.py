@@ -105,6 +105,24 @@ def test_host_cluster_bit_exact_vs_oracle(sr, oracle, seed):
         np.testing.assert_array_equal(got2, ref)
 
 
+@pytest.mark.parametrize("seed", [5, 6, 7])
+def test_host_cluster_reinserts_and_zero_similarity_pairs(sr, oracle, seed):
+    """The library's Alg 3 keeps re-inserted pairs with J = 0 apart from the heap and proves
+    J = 0 from row digests: compare with the oracle's plain priority queue on matrices where
+    most re-inserts have J = 0 (power-law-ish columns, many clusters), and with caller-given
+    candidates that include J = 0 pairs (allowed by sr_host_cluster, never made by the LSH)."""
+    rng = np.random.default_rng(seed)
+    A = g.random_csr(3000, 4000, 0.002, seed, empty_frac=0.1)
+    E = oracle.candidates(A.rowptr, A.colidx, 32, 2, 4, 8)
+    extra = rng.integers(0, 3000, size=(400, 2))
+    E2 = oracle.pack_pairs([(int(i), int(j)) for i, j in extra if i != j] +
+                           [(int(e) >> 32, int(e) & 0xFFFFFFFF) for e in E])
+    for pairs in (E, E2):
+        for thr in (3, 16, 256):
+            ref = oracle.cluster(A.rowptr, A.colidx, pairs, thr)
+            np.testing.assert_array_equal(sr.host_cluster(A.rowptr, A.colidx, pairs, thr), ref)
+
+
 def test_host_cluster_fig6(sr):
     A = g.fig1a()
     from oracle import oracle as O
