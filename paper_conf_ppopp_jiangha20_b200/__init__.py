@@ -145,11 +145,33 @@ def _ptr(t) -> C.c_void_p:
     return C.c_void_p(int(t.data_ptr()))
 
 
-def _stream(stream):
+def _stream(stream, device: int | None = None):
+    """cudaStream_t of `stream`; None = torch's current stream of `device` (the matrix's GPU)."""
     if stream is None:
         import torch
-        stream = torch.cuda.current_stream()
+        stream = torch.cuda.current_stream(device)
     return C.c_void_p(int(stream.cuda_stream))
+
+
+def _check_dense(name: str, T, rows: int, device: int, K: int | None = None, contiguous: bool = False):
+    """The C ABI receives only pointers and leading dimensions, so the binding checks what the
+    kernels will read or write: fp32, CUDA, this matrix's device, 2-D with unit column stride
+    (or contiguous 1-D), and the row count the operation indexes."""
+    import torch
+    if T.dtype != torch.float32 or not T.is_cuda:
+        raise ValueError(f"{name} must be an fp32 CUDA tensor")
+    if T.device.index != device:
+        raise ValueError(f"{name} is on cuda:{T.device.index}, the matrix on cuda:{device}")
+    if contiguous:
+        if T.dim() != 1 or not T.is_contiguous() or T.numel() != rows:
+            raise ValueError(f"{name} must be a contiguous 1-D tensor of {rows} values")
+        return
+    if T.dim() != 2 or T.stride(1) != 1 or T.stride(0) < T.shape[1]:
+        raise ValueError(f"{name} must be 2-D with unit column stride and row stride >= its width")
+    if T.shape[0] != rows:
+        raise ValueError(f"{name} has {T.shape[0]} rows, expected {rows}")
+    if K is not None and T.shape[1] != K:
+        raise ValueError(f"{name} has {T.shape[1]} columns, expected K = {K}")
 
 
 class SparseMatrix:
@@ -292,37 +314,36 @@ class SparseMatrix:
 
     # -- compute (torch tensors on this matrix's device; asynchronous on `stream`)
     def spmm(self, B, C_out=None, stream=None):
-        """C := A·B (Alg 1).  B: [ncols, K] fp32 CUDA tensor (row stride >= K)."""
+        """C := A·B (Alg 1).  B: [ncols, K] fp32 CUDA tensor on this matrix's device (row stride
+        >= K); C_out: [out_rows, K] (row stride >= K) or None."""
         import torch
-        if B.dtype != torch.float32 or not B.is_cuda or B.dim() != 2 or B.stride(1) != 1:
-            raise ValueError("B must be a 2-D fp32 CUDA tensor with unit column stride")
+        _check_dense("B", B, self.ncols, self.device)
         K = B.shape[1]
         if C_out is None:
             C_out = torch.empty((self.out_rows, K), dtype=torch.float32, device=B.device)
-        _check(lib().sr_spmm(self._h, _ptr(B), K, B.stride(0), _ptr(C_out), C_out.stride(0), _stream(stream)))
+        _check_dense("C_out", C_out, self.out_rows, self.device, K)
+        _check(lib().sr_spmm(self._h, _ptr(B), K, B.stride(0), _ptr(C_out), C_out.stride(0),
+                             _stream(stream, self.device)))
         return C_out
 
     def set_values(self, vals, stream=None):
         """Replace the nonzero values the kernels use (sr_set_values): fp32 CUDA tensor of
         out_nnz values in the order sddmm() writes."""
-        import torch
-        if vals.dtype != torch.float32 or not vals.is_cuda or vals.numel() != self.out_nnz or not vals.is_contiguous():
-            raise ValueError("vals must be a contiguous fp32 CUDA tensor of out_nnz values")
-        _check(lib().sr_set_values(self._h, _ptr(vals), _stream(stream)))
+        _check_dense("vals", vals, self.out_nnz, self.device, contiguous=True)
+        _check(lib().sr_set_values(self._h, _ptr(vals), _stream(stream, self.device)))
 
     def sddmm(self, X, Y, out=None, stream=None):
-        """out[p] := vals[p]·<X[row(p)], Y[col(p)]> (Alg 2) in the caller's nnz order."""
+        """out[p] := vals[p]·<X[row(p)], Y[col(p)]> (Alg 2) in the caller's nnz order.
+        X: [nrows, K], Y: [ncols, K] fp32 CUDA tensors; out: contiguous [out_nnz] or None."""
         import torch
-        for T in (X, Y):
-            if T.dtype != torch.float32 or not T.is_cuda or T.dim() != 2 or T.stride(1) != 1:
-                raise ValueError("X, Y must be 2-D fp32 CUDA tensors with unit column stride")
+        _check_dense("X", X, self.nrows, self.device)
         K = X.shape[1]
-        if Y.shape[1] != K:
-            raise ValueError("X and Y need the same K")
+        _check_dense("Y", Y, self.ncols, self.device, K)
         if out is None:
             out = torch.empty(self.out_nnz, dtype=torch.float32, device=X.device)
+        _check_dense("out", out, self.out_nnz, self.device, contiguous=True)
         _check(lib().sr_sddmm(self._h, _ptr(X), X.stride(0), _ptr(Y), Y.stride(0), K, _ptr(out),
-                              _stream(stream)))
+                              _stream(stream, self.device)))
         return out
 
 
@@ -348,8 +369,12 @@ def trial(cands, op: str, U, V=None, out=None, reps: int = 5, stream=None):
         raise ValueError("op must be 'spmm' or 'sddmm'")
     best = C.c_int32()
     ms = (C.c_float * n)()
+    dev = cands[0].device
+    _check_dense("U", U, cands[0].ncols if op == "spmm" else cands[0].nrows, dev)
+    if op == "sddmm":
+        _check_dense("V", V, cands[0].ncols, dev, K)
     _check(lib().sr_trial(C.cast(hs, C.c_void_p), n, code, _ptr(U), U.stride(0), pv, ldv, K, _ptr(out), ldo, reps,
-                          _stream(stream), C.byref(best), C.cast(ms, C.c_void_p)))
+                          _stream(stream, dev), C.byref(best), C.cast(ms, C.c_void_p)))
     return best.value, [float(x) for x in ms]
 
 
@@ -380,13 +405,13 @@ def host_partition(weights, G: int) -> np.ndarray:
 def scatter_rows(src, rows, dst, stream=None):
     """dst[rows[r]] = src[r] on the device (rows: int32 CUDA tensor; -1 entries skipped)."""
     _check(lib().sr_scatter_rows(_ptr(src), src.stride(0), _ptr(rows), rows.numel(), src.shape[1], _ptr(dst),
-                                 dst.stride(0), _stream(stream)))
+                                 dst.stride(0), _stream(stream, dst.device.index)))
     return dst
 
 
 def scatter_values(src, ids, dst, stream=None):
     """dst[ids[i]] = src[i] on the device (ids: int64 CUDA tensor; -1 entries skipped)."""
-    _check(lib().sr_scatter_values(_ptr(src), _ptr(ids), ids.numel(), _ptr(dst), _stream(stream)))
+    _check(lib().sr_scatter_values(_ptr(src), _ptr(ids), ids.numel(), _ptr(dst), _stream(stream, dst.device.index)))
     return dst
 
 

@@ -213,40 +213,66 @@ int build_identity_plan(sr_csr_s* h, cudaStream_t s) {
   return SR_OK;
 }
 
-// Device plan of a (possibly sharded) tiling.
+// Device plan of a (possibly sharded) tiling.  Built into fresh buffers and installed only when
+// every upload and the final synchronisation succeeded, so a failure (ENOMEM, a CUDA error)
+// leaves the handle's previous plan intact.
+int build_exec_plan_into(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s, DevPlan& P,
+                         std::vector<int32_t>& shard_rows, std::vector<int64_t>& shard_nnz_ids);
+
 int build_exec_plan(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s) {
+  DevPlan P;
+  std::vector<int32_t> rows;
+  std::vector<int64_t> ids;
+  const int rc = build_exec_plan_into(h, pb, pe, s, P, rows, ids);
+  if (rc != SR_OK) {
+    cudaStreamSynchronize(s);  // no copy into P's buffers may still be in flight when they are freed
+    cudaGetLastError();
+    return rc;
+  }
+  for (int i = 0; i < 8; ++i) {  // the profiling events belong to the handle
+    P.ev[i] = h->plan.ev[i];
+    h->plan.ev[i] = nullptr;
+  }
+  P.profiling = h->plan.profiling;
+  h->plan = std::move(P);
+  h->shard_rows = std::move(rows);
+  h->shard_nnz_ids = std::move(ids);
+  return SR_OK;
+}
+
+int build_exec_plan_into(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s, DevPlan& P,
+                         std::vector<int32_t>& shard_rows, std::vector<int64_t>& shard_nnz_ids) {
   const HostCSR& A = h->A;
   const Tiling& T = h->tiles;
-  DevPlan& P = h->plan;
   const int64_t M = A.M;
   const int32_t PR = h->params.panel_rows;
   const bool sharded = h->params.world > 1;
   const int64_t q0s = std::min<int64_t>(M, pb * PR), q1s = std::min<int64_t>(M, pe * PR);
   const std::vector<int32_t>& perm1 = h->perm1;
   // shard rows / packed nnz order: by position, dense (slot order) then remainder (CSR order)
-  h->shard_rows.assign(perm1.begin() + q0s, perm1.begin() + q1s);
+  shard_rows.assign(perm1.begin() + q0s, perm1.begin() + q1s);
   std::vector<int32_t> d_out((size_t)T.n_dense(), 0), r_out(T.r_col.size(), 0);
-  h->shard_nnz_ids.clear();
+  shard_nnz_ids.clear();
   {
     int64_t k = 0;
     for (int64_t q = q0s; q < q1s; ++q) {
       for (int64_t e = T.drow_ptr[q]; e < T.drow_ptr[q + 1]; ++e) {
         const int64_t orig = A.identity_pos ? T.d_cidx[e] : A.opos[T.d_cidx[e]];
         d_out[e] = (int32_t)(sharded ? k : orig);
-        h->shard_nnz_ids.push_back(orig);
+        shard_nnz_ids.push_back(orig);
         ++k;
       }
       for (int64_t e = T.rrow_ptr[q]; e < T.rrow_ptr[q + 1]; ++e) {
         const int64_t orig = A.identity_pos ? T.r_cidx[e] : A.opos[T.r_cidx[e]];
         r_out[e] = (int32_t)(sharded ? k : orig);
-        h->shard_nnz_ids.push_back(orig);
+        shard_nnz_ids.push_back(orig);
         ++k;
       }
     }
   }
   if (!sharded) {  // single shard: outputs come back in the caller's order
-    std::iota(h->shard_rows.begin(), h->shard_rows.end(), 0);
-    std::iota(h->shard_nnz_ids.begin(), h->shard_nnz_ids.end(), 0);
+    std::iota(shard_rows.begin(), shard_rows.end(), 0);
+    std::iota(shard_nnz_ids.begin(), shard_nnz_ids.end(), 0);
   }
   // phase D: execution tiles of <= kMaxExecTile dense columns (the plan's tiles of tile_cols
   // columns are reported in the metadata and staged in sub-tiles); each tile's entries are
@@ -481,6 +507,28 @@ int reorder_round(const int64_t* rowptr, const int32_t* col, int64_t M, const sr
   return SR_OK;
 }
 
+// Restores a handle's plan state (parameters, orders, tiling, stats) unless committed: a failed
+// sr_reorder / sr_plan_load leaves the handle as it was (its identity plan stays usable).
+struct PlanRollback {
+  sr_csr_s* h;
+  bool armed = true;
+  sr_reorder_params params;
+  std::vector<int32_t> perm1, perm2;
+  Tiling tiles;
+  sr_plan_stats stats;
+  explicit PlanRollback(sr_csr_s* h_)
+      : h(h_), params(h_->params), perm1(h_->perm1), perm2(h_->perm2), tiles(h_->tiles), stats(h_->stats) {}
+  ~PlanRollback() {
+    if (!armed) return;
+    h->params = params;
+    h->perm1 = std::move(perm1);
+    h->perm2 = std::move(perm2);
+    h->tiles = std::move(tiles);
+    h->stats = stats;
+  }
+  void commit() { armed = false; }
+};
+
 // Shard selection + device execution plan of the plan held in h (perm1, its tiling, perm2).
 int finish_plan(sr_csr_s* h, cudaStream_t s) {
   const sr_reorder_params* p = &h->params;
@@ -640,6 +688,7 @@ int sr_reorder(sr_csr h, const sr_reorder_params* p, sr_stream stream) {
   DeviceGuard dg(h->device);
   cudaStream_t s = stream ? (cudaStream_t)stream : h->init_stream;
   const double t_start = now_s();
+  PlanRollback rollback(h);
   h->params = *p;
   const HostCSR& A = h->A;
   const int64_t M = A.M, nnz = A.nnz();
@@ -696,6 +745,7 @@ int sr_reorder(sr_csr h, const sr_reorder_params* p, sr_stream stream) {
   st.n_perm2 = (int64_t)h->perm2.size();
   SR_TRY(finish_plan(h, s));
   st.t_total_s = now_s() - t_start;
+  rollback.commit();
   return SR_OK;
 }
 
@@ -1014,6 +1064,7 @@ int sr_plan_load(sr_csr h, const void* buf, int64_t len, int32_t world, int32_t 
   }
   DeviceGuard dg(h->device);
   cudaStream_t s = stream ? (cudaStream_t)stream : h->init_stream;
+  PlanRollback rollback(h);
   h->params = p;
   const double t0 = now_s();
   Tiling T;
@@ -1023,16 +1074,11 @@ int sr_plan_load(sr_csr h, const void* buf, int64_t len, int32_t world, int32_t 
     int64_t nonempty = 0;
     for (int64_t q = 0; q < M; ++q) nonempty += T.rrow_ptr[q + 1] > T.rrow_ptr[q];
     for (int32_t q : perm2) {
-      if (q < 0 || q >= M || seen[q] || T.rrow_ptr[q + 1] == T.rrow_ptr[q]) {
-        sr_default_params(&h->params);
+      if (q < 0 || q >= M || seen[q] || T.rrow_ptr[q + 1] == T.rrow_ptr[q])
         return einval("sr_plan_load: perm2 does not match the tiling of perm1");
-      }
       seen[q] = 1;
     }
-    if (nonempty != len2) {
-      sr_default_params(&h->params);
-      return einval("sr_plan_load: perm2 does not match the tiling of perm1");
-    }
+    if (nonempty != len2) return einval("sr_plan_load: perm2 does not match the tiling of perm1");
   }
   h->perm1 = std::move(perm1);
   h->perm2 = std::move(perm2);
@@ -1042,6 +1088,7 @@ int sr_plan_load(sr_csr h, const void* buf, int64_t len, int32_t world, int32_t 
   h->stats = st;
   SR_TRY(finish_plan(h, s));
   h->stats.t_total_s = now_s() - t_start;
+  rollback.commit();
   return SR_OK;
 }
 

@@ -26,6 +26,7 @@
 #include <parallel/algorithm>
 #include <queue>
 #include <cstring>
+#include <memory>
 #include <numeric>
 #include <vector>
 
@@ -96,9 +97,9 @@ class PairSet {
   explicit PairSet(size_t expected) {
     size_t cap = 16;
     while (cap < 2 * expected + 16) cap <<= 1;
-    slots_.assign(cap, kEmpty);
-    mask_ = cap - 1;
+    reset(cap);
   }
+  void prefetch(uint64_t k) const { __builtin_prefetch(&slots_[hash(k) & mask_]); }
   bool contains(uint64_t k) const {
     size_t h = hash(k) & mask_;
     while (true) {
@@ -119,7 +120,7 @@ class PairSet {
   }
   void set_size(size_t n) { size_ = n; }
   void insert(uint64_t k) {
-    if (2 * (size_ + 1) > slots_.size()) grow();
+    if (2 * (size_ + 1) > cap_) grow();
     size_t h = hash(k) & mask_;
     while (slots_[h] != kEmpty) {
       if (slots_[h] == k) return;
@@ -139,17 +140,24 @@ class PairSet {
     k ^= k >> 33;
     return (size_t)k;
   }
-  void grow() {
-    std::vector<uint64_t> old;
-    old.swap(slots_);
-    slots_.assign(old.size() * 2, kEmpty);
-    mask_ = slots_.size() - 1;
-    size_ = 0;
-    for (uint64_t v : old)
-      if (v != kEmpty) insert(v);
+  void reset(size_t cap) {  // uninitialised allocation + parallel first-touch fill
+    slots_.reset(new uint64_t[cap]);
+    cap_ = cap;
+    mask_ = cap - 1;
+    uint64_t* sl = slots_.get();
+#pragma omp parallel for schedule(static)
+    for (int64_t k = 0; k < (int64_t)cap; ++k) sl[k] = kEmpty;
   }
-  std::vector<uint64_t> slots_;
-  size_t mask_ = 0, size_ = 0;
+  void grow() {
+    std::unique_ptr<uint64_t[]> old = std::move(slots_);
+    const size_t ocap = cap_;
+    reset(2 * ocap);
+    size_ = 0;
+    for (size_t k = 0; k < ocap; ++k)
+      if (old[k] != kEmpty) insert(old[k]);
+  }
+  std::unique_ptr<uint64_t[]> slots_;
+  size_t cap_ = 0, mask_ = 0, size_ = 0;
 };
 
 inline void intersect(const int64_t* rowptr, const int32_t* col, int64_t a, int64_t b,
@@ -212,7 +220,8 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
   double t0 = now();
   // initial candidates in heap order; the heap order is a strict total order (R10), so any
   // sort gives the same array
-  std::vector<Cand> init((size_t)npairs);
+  std::unique_ptr<Cand[]> init_buf(new Cand[(size_t)npairs]);  // filled below (no zeroing pass)
+  Cand* const init = init_buf.get();
   // membership (line 27, R9): one open-addressing hash set of the initial candidates and the
   // re-inserted pairs (one cache miss per lookup); above 2^26 candidates the initial ones are
   // found by binary search in the key-sorted pair array instead (memory), if the caller has it
@@ -264,7 +273,7 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
   bool sorted = true;
   for (int64_t e = 1; e < npairs && sorted; ++e) sorted = !before(init[e], init[e - 1]);
   const double t1 = now();
-  if (!sorted) __gnu_parallel::sort(init.begin(), init.end(), before);
+  if (!sorted) __gnu_parallel::sort(init, init + npairs, before);
   const double t2 = now();
   int64_t n_reinsert = 0, n_zero = 0;
 
@@ -307,7 +316,7 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
   while (init_pos > 0 && init[init_pos - 1].inter == 0) --init_pos;
   size_t cur = 0, zc = 0;
   int64_t nclusters = M;
-  constexpr size_t PF = 32, PF2 = 12;  // prefetch distances over the initial-candidate cursor
+  constexpr size_t PF = 32, PF2 = 16, PF3 = 8;  // prefetch distances over the initial-candidate cursor
   while (nclusters > 0) {
     int32_t i, j;
     if (!zero_phase) {
@@ -320,6 +329,21 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
           __builtin_prefetch(&nd[nd[init[cur + PF2].i].parent]);
           __builtin_prefetch(&nd[nd[init[cur + PF2].j].parent]);
         }
+        if (cur + PF3 < init_pos) {
+          // third level: a nearer pair's likely roots (read-only walk, merges are rare between
+          // here and its pop), whose membership slot and digests the else branch will read
+          int32_t a = (int32_t)init[cur + PF3].i, b = (int32_t)init[cur + PF3].j;
+          if (nd[a].parent != a || nd[b].parent != b) {
+            for (int k = 0; k < 4 && nd[a].parent != a; ++k) a = nd[a].parent;
+            for (int k = 0; k < 4 && nd[b].parent != b; ++k) b = nd[b].parent;
+            if (a != b) {
+              const uint64_t key = ((uint64_t)std::min(a, b) << 32) | (uint64_t)std::max(a, b);
+              if (!by_key) members.prefetch(key);
+              __builtin_prefetch(&dig[a]);
+              __builtin_prefetch(&dig[b]);
+            }
+          }
+        }
         i = (int32_t)init[cur].i;
         j = (int32_t)init[cur].j;
         ++cur;
@@ -330,7 +354,7 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
       } else {
         zero_phase = true;
         if (dbg) fprintf(stderr, "  J>0 phase %.3f s, %lld clusters left, %zu J=0 pairs\n", now() - t2, (long long)nclusters, zero_keys.size());
-        for (size_t e = init_pos; e < init.size(); ++e) zero_keys.push_back(((uint64_t)init[e].i << 32) | init[e].j);
+        for (size_t e = init_pos; e < (size_t)npairs; ++e) zero_keys.push_back(((uint64_t)init[e].i << 32) | init[e].j);
         __gnu_parallel::sort(zero_keys.begin(), zero_keys.end());
         continue;
       }

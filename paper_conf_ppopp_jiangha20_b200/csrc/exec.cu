@@ -16,6 +16,9 @@
 #include <cudaTypedefs.h>  // PFN_cuTensorMapEncodeTiled
 
 #include <algorithm>
+#include <cstring>
+#include <map>
+#include <mutex>
 
 #include "internal.h"
 
@@ -992,6 +995,37 @@ bool make_row_gather_map(CUtensorMap* map, const float* base, int64_t rows, int6
                 CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// Per-handle cache of the tensor map (encoded once per operand base / shape, not per call) and a
+// process-wide record of the kernels whose dynamic shared-memory limit has been raised on a
+// device, so a steady-state sr_spmm / sr_sddmm call does launch work only.
+bool cached_row_gather_map(DevPlan& P, CUtensorMap* map, const float* base, int64_t rows, int64_t K, int64_t ld,
+                           int box_cols) {
+  static_assert(sizeof(CUtensorMap) <= sizeof(P.tmap_bytes), "tensor map cache too small");
+  TmapKey key{base, rows, K, ld, box_cols};
+  if (!(P.tmap_valid && P.tmap_key == key)) {
+    CUtensorMap m;
+    P.tmap_ok = make_row_gather_map(&m, base, rows, K, ld, box_cols);
+    std::memcpy(P.tmap_bytes, &m, sizeof(m));
+    P.tmap_key = key;
+    P.tmap_valid = true;
+  }
+  std::memcpy(map, P.tmap_bytes, sizeof(CUtensorMap));
+  return P.tmap_ok;
+}
+
+int raise_smem_limit(const void* kern, size_t smem) {
+  static std::mutex mu;
+  static std::map<std::pair<const void*, int>, size_t> done;
+  int dev = 0;
+  SR_CUDA_TRY(cudaGetDevice(&dev));
+  std::lock_guard<std::mutex> lock(mu);
+  size_t& cur = done[{kern, dev}];
+  if (cur >= smem) return SR_OK;
+  SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  cur = smem;
+  return SR_OK;
+}
+
 // Phase-S kernel choice (measurement knob SR_PHASE_S; profiles/r01/NOTES.md, profiles/r02/NOTES.md):
 // 1 (default) = row-group task kernels where K allows them, 0 = one-row-per-warp kernels (also
 // the path for K that is not a multiple of 32).
@@ -1027,7 +1061,7 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
     const size_t smem =
         StageLayout{((TW + 3) & ~3) * KC, P.trp_stride, false, kSpmmStages, 0, true}.smem(kSpmmStages);
     CUtensorMap tmap;
-    const int use_tmap = (VEC == 4 && make_row_gather_map(&tmap, B, h->A.N, K, ldb, KC)) ? 1 : 0;
+    const int use_tmap = (VEC == 4 && cached_row_gather_map(P, &tmap, B, h->A.N, K, ldb, KC)) ? 1 : 0;
     if (P.n_dslots > 0 && P.dscratch_k < K) {
       SR_TRY(P.dscratch.alloc((size_t)P.n_dslots * P.panel_rows * K));
       P.dscratch_k = K;
@@ -1035,7 +1069,7 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
     const unsigned grid = (unsigned)std::min<int64_t>(P.n_units, (int64_t)kDenseCtasPerSM * num_sms());
     const int flags = (VEC == 4 ? 1 : 0) | (dense_dbg() << 1);
     auto launch = [&](auto kern) -> int {
-      SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+      SR_TRY(raise_smem_limit(reinterpret_cast<const void*>(kern), smem));
       kern<<<grid, (kDenseWarps + 1) * 32, smem, s>>>(
           P.units.p, (int)P.n_units, P.vtiles.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.dense_out.p, B, ldb, C, ldc,
           (int)K, TW, P.trp_stride, P.panel_rows, P.dscratch.p, P.dsplit_info.p, P.dsplit_counter.p, P.blobs.p,
@@ -1104,11 +1138,11 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
     const size_t smem =
         StageLayout{((TW + 3) & ~3) * NCH_D * KC, P.trp_stride, true, kSddmmStages, 0, true}.smem(kSddmmStages);
     CUtensorMap tmap;
-    const int use_tmap = (VEC == 4 && make_row_gather_map(&tmap, Y, h->A.N, K, ldy, NCH_D * KC)) ? 1 : 0;
+    const int use_tmap = (VEC == 4 && cached_row_gather_map(P, &tmap, Y, h->A.N, K, ldy, NCH_D * KC)) ? 1 : 0;
     const unsigned grid = (unsigned)std::min<int64_t>(P.n_units, (int64_t)kDenseCtasPerSM * num_sms());
     const int flags = (VEC == 4 ? 1 : 0) | (dense_dbg() << 1);
     auto launch = [&](auto kern) -> int {
-      SR_CUDA_TRY(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+      SR_TRY(raise_smem_limit(reinterpret_cast<const void*>(kern), smem));
       kern<<<grid, (kDenseWarps + 1) * 32, smem, s>>>(
           P.units.p, (int)P.n_units, P.vtiles.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.d_oidx.p, P.pos_xrow.p, X, ldx,
           Y, ldy, (int)K, TW, P.trp_stride, out, P.blobs.p, P.blob_meta.p, tmap, use_tmap, flags);

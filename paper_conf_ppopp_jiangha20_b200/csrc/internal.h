@@ -41,6 +41,17 @@ struct DevBuf {
   DevBuf() = default;
   DevBuf(const DevBuf&) = delete;
   DevBuf& operator=(const DevBuf&) = delete;
+  DevBuf(DevBuf&& o) noexcept : p(o.p), n(o.n) { o.p = nullptr; o.n = 0; }
+  DevBuf& operator=(DevBuf&& o) noexcept {
+    if (this != &o) {
+      release();
+      p = o.p;
+      n = o.n;
+      o.p = nullptr;
+      o.n = 0;
+    }
+    return *this;
+  }
   ~DevBuf() { release(); }
   void release() {
     if (p) cudaFree(p);
@@ -129,8 +140,21 @@ constexpr int kMaxTileEntries = 384;  // SpMM: 3 stages + blob ring must fit twi
 // producer-side record of a unit: DUnit, its VTiles, its dense column ids (16-byte aligned)
 constexpr int kMaxUnitBlobBytes = 32 + kMaxUnitTiles * 16 + kMaxUnitTiles * kMaxExecTile * 4;
 
+struct TmapKey {
+  const void* base = nullptr;
+  int64_t rows = 0, K = 0, ld = 0;
+  int box = 0;
+  bool operator==(const TmapKey& o) const {
+    return base == o.base && rows == o.rows && K == o.K && ld == o.ld && box == o.box;
+  }
+};
+
 // Device-resident execution plan.
 struct DevPlan {
+  // cached TMA tensor map of the last phase-D operand (exec.cu: cached_row_gather_map)
+  alignas(64) unsigned char tmap_bytes[128] = {};
+  TmapKey tmap_key;
+  bool tmap_valid = false, tmap_ok = false;
   // phase D
   DevBuf<DUnit> units;
   int64_t n_units = 0;

@@ -214,6 +214,31 @@ def test_strided_and_misaligned_operands(env, oracle):
     assert torch.all(C1[:, K:] == 7.0)  # padding columns untouched
 
 
+def test_binding_rejects_bad_operands(env):
+    """The C ABI sees only pointers and leading dimensions: the binding must refuse operands the
+    kernels would read or write out of bounds or scramble."""
+    sr, torch = env
+    A = g.random_csr(50, 40, 0.1, 3)
+    M = sr.SparseMatrix.from_csr(A)
+    K = 8
+    B = torch.ones((40, K), device="cuda")
+    X, Y = torch.ones((50, K), device="cuda"), torch.ones((40, K), device="cuda")
+    bad = [lambda: M.spmm(torch.ones((39, K), device="cuda")),                      # too few B rows
+           lambda: M.spmm(B.double()),                                             # dtype
+           lambda: M.spmm(B.cpu()),                                                # host tensor
+           lambda: M.spmm(B, torch.empty((49, K), device="cuda")),                 # C too small
+           lambda: M.spmm(B, torch.empty((50, 2 * K), device="cuda")[:, ::2]),     # C column stride 2
+           lambda: M.spmm(B.t().contiguous().t()),                                 # B column stride != 1
+           lambda: M.sddmm(torch.ones((49, K), device="cuda"), Y),                 # X rows
+           lambda: M.sddmm(X, torch.ones((40, K + 1), device="cuda")),             # K mismatch
+           lambda: M.sddmm(X, Y, torch.empty(2 * A.nnz, device="cuda")[::2]),      # out not contiguous
+           lambda: M.set_values(torch.ones(A.nnz - 1, device="cuda"))]             # value count
+    for f in bad:
+        with pytest.raises(ValueError):
+            f()
+    torch.cuda.synchronize()
+
+
 def test_empty_and_degenerate(env, oracle):
     sr, torch = env
     # all rows empty
