@@ -475,10 +475,11 @@ def build_plan(sr, A, params, world, rank, local_rank):
     its shard.  Returns (handle, reorder seconds on rank 0, stats of the full plan, image,
     shard load seconds)."""
     import torch
-    t0 = time.perf_counter()
     full, st_full, image = None, None, None
+    t0 = time.perf_counter()
     if rank == 0:
-        full = sr.SparseMatrix.from_csr(A, device=local_rank)
+        full = sr.SparseMatrix.from_csr(A, device=local_rank)  # ingest (a1) is not preprocessing
+        t0 = time.perf_counter()
         full.reorder(params)
         st_full = full.stats()
         if world > 1:
@@ -708,6 +709,7 @@ def run_ours(args, A, ops, rank, world, local_rank):
             "extra_K": extra,
             "preprocess": {"seconds": t_pre, "lsh1_s": stp["t_lsh1_s"], "cluster1_s": stp["t_cluster1_s"],
                            "tile_s": stp["t_tile_s"], "lsh2_s": stp["t_lsh2_s"], "cluster2_s": stp["t_cluster2_s"],
+                           "plan_build_s": stp["t_plan_s"],
                            "round1": stp["round1"], "round2": stp["round2"], "E1": stp["E1"], "E2": stp["E2"],
                            "dense_ratio0": stp["dense0"] / max(1, stp["nnz"]),
                            "dense_ratio": stp["dense1"] / max(1, stp["nnz"]),

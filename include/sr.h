@@ -49,7 +49,8 @@ typedef struct sr_csr_s* sr_csr;       /* opaque handle owned by the library */
  * Deep-copies (the caller keeps its arrays).  Rows need not be column-sorted:
  * they are sorted internally and SDDMM results still come back in the caller's
  * nnz order (R22).  The handle starts with the identity plan (no tiles): spmm /
- * sddmm work right away as the plain row-wise kernels of P:101.
+ * sddmm work right away as the plain row-wise kernels of P:101 (its device arrays are built on
+ * the first spmm / sddmm / set_values call, synchronously, unless a plan is installed first).
  * Errors: SR_EINVAL (malformed / duplicates), SR_EUNSUPPORTED, SR_ENOMEM, SR_ECUDA.
  * ---------------------------------------------------------------------------*/
 int sr_csr_create(int64_t nrows, int64_t ncols, int64_t nnz, const int64_t* rowptr,
@@ -211,6 +212,7 @@ typedef struct {
   int64_t shard_panel_begin, shard_panel_end; /* panels owned by this handle             */
   int64_t shard_nrows, shard_nnz;
   double t_lsh1_s, t_cluster1_s, t_tile_s, t_lsh2_s, t_cluster2_s, t_total_s; /* wall time */
+  double t_plan_s;       /* wall time of the device execution plan build (tasks, uploads)  */
 } sr_plan_stats;
 
 int sr_get_plan_stats(sr_csr h, sr_plan_stats* out);

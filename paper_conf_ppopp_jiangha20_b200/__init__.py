@@ -48,7 +48,8 @@ class PlanStats(C.Structure):
                 ("n_perm2", C.c_int64), ("shard_panel_begin", C.c_int64), ("shard_panel_end", C.c_int64),
                 ("shard_nrows", C.c_int64), ("shard_nnz", C.c_int64),
                 ("t_lsh1_s", C.c_double), ("t_cluster1_s", C.c_double), ("t_tile_s", C.c_double),
-                ("t_lsh2_s", C.c_double), ("t_cluster2_s", C.c_double), ("t_total_s", C.c_double)]
+                ("t_lsh2_s", C.c_double), ("t_cluster2_s", C.c_double), ("t_total_s", C.c_double),
+                ("t_plan_s", C.c_double)]
 
     def as_dict(self) -> dict:
         return {k: getattr(self, k) for k, _ in self._fields_}

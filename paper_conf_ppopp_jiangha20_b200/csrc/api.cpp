@@ -74,27 +74,32 @@ struct ItemBuilder {
 // column load it once (access model O14 / P:111); distinct columns = compulsory.
 void sparse_traffic(const ItemBuilder& ib, int64_t n_nonzero, int64_t n_zero, const std::vector<int2>& ent,
                     int64_t N, sr_traffic_model& t) {
-  std::vector<int64_t> mark((size_t)N, -1);
   std::vector<uint8_t> seen((size_t)N, 0);
-  int64_t loads = 0, distinct = 0, nnz = 0, rows = 0;
-  for (int64_t it = 0; it < n_nonzero; ++it) {
-    const int64_t grp = it / 8;
-    const Item& x = ib.items[it];
-    nnz += x.e1 - x.e0;
-    const uint32_t m = ib.meta[it];
-    if (!(m & kItemSplit) || (m & kItemSlotMask) == (uint32_t)ib.split_info[m & kItemSlotMask].x) ++rows;
-    for (int32_t e = x.e0; e < x.e1; ++e) {
-      const int32_t c = ent[e].x;
-      if (mark[c] != grp) {
-        mark[c] = grp;
-        ++loads;
+  int64_t loads = 0, nnz = 0, rows = 0;
+  const int64_t ngroups = (n_nonzero + 7) / 8;
+#pragma omp parallel reduction(+ : loads, nnz, rows)
+  {
+    std::vector<int32_t> cols;
+#pragma omp for schedule(dynamic, 1024)
+    for (int64_t grp = 0; grp < ngroups; ++grp) {
+      cols.clear();
+      for (int64_t it = grp * 8; it < std::min(n_nonzero, grp * 8 + 8); ++it) {
+        const Item& x = ib.items[it];
+        nnz += x.e1 - x.e0;
+        const uint32_t m = ib.meta[it];
+        if (!(m & kItemSplit) || (m & kItemSlotMask) == (uint32_t)ib.split_info[m & kItemSlotMask].x) ++rows;
+        for (int32_t e = x.e0; e < x.e1; ++e) {
+          cols.push_back(ent[e].x);
+          __atomic_store_n(&seen[ent[e].x], (uint8_t)1, __ATOMIC_RELAXED);
+        }
       }
-      if (!seen[c]) {
-        seen[c] = 1;
-        ++distinct;
-      }
+      std::sort(cols.begin(), cols.end());
+      loads += std::unique(cols.begin(), cols.end()) - cols.begin();
     }
   }
+  int64_t distinct = 0;
+#pragma omp parallel for reduction(+ : distinct) schedule(static)
+  for (int64_t c = 0; c < N; ++c) distinct += seen[c];
   t.sparse_nnz = nnz;
   t.sparse_items = n_nonzero + n_zero;
   t.sparse_rows = rows;
@@ -213,6 +218,14 @@ int build_identity_plan(sr_csr_s* h, cudaStream_t s) {
   return SR_OK;
 }
 
+// The identity plan on first use of a handle without a reordered plan.  Synchronous (once).
+int ensure_plan(sr_csr_s* h) {
+  if (h->reordered || h->identity_ready) return SR_OK;
+  SR_TRY(build_identity_plan(h, h->init_stream));
+  h->identity_ready = true;
+  return SR_OK;
+}
+
 // Device plan of a (possibly sharded) tiling.  Built into fresh buffers and installed only when
 // every upload and the final synchronisation succeeded, so a failure (ENOMEM, a CUDA error)
 // leaves the handle's previous plan intact.
@@ -253,7 +266,14 @@ int build_exec_plan_into(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s, De
   shard_rows.assign(perm1.begin() + q0s, perm1.begin() + q1s);
   std::vector<int32_t> d_out((size_t)T.n_dense(), 0), r_out(T.r_col.size(), 0);
   shard_nnz_ids.clear();
-  {
+  if (!sharded) {  // outputs in the caller's order: every index is the caller's own position
+    const int64_t nd = T.n_dense(), nr = (int64_t)T.r_col.size();
+#pragma omp parallel for schedule(static)
+    for (int64_t e = 0; e < nd; ++e) d_out[e] = (int32_t)(A.identity_pos ? T.d_cidx[e] : A.opos[T.d_cidx[e]]);
+#pragma omp parallel for schedule(static)
+    for (int64_t e = 0; e < nr; ++e) r_out[e] = (int32_t)(A.identity_pos ? T.r_cidx[e] : A.opos[T.r_cidx[e]]);
+    shard_nnz_ids.resize((size_t)(nd + nr));
+  } else {
     int64_t k = 0;
     for (int64_t q = q0s; q < q1s; ++q) {
       for (int64_t e = T.drow_ptr[q]; e < T.drow_ptr[q + 1]; ++e) {
@@ -416,19 +436,29 @@ int build_exec_plan_into(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s, De
   se.reserve(T.r_col.size());
   so.reserve(T.r_col.size());
   ItemBuilder ib;
+  std::vector<int32_t> rows_s;  // the shard's remainder positions in perm2 order
+  std::vector<int64_t> soff;    // their offsets in the stream
+  int64_t ns = 0;
   for (int32_t q : h->perm2) {
     if (q < q0s || q >= q1s) continue;
-    const int32_t e0 = (int32_t)se.size();
-    for (int64_t e = T.rrow_ptr[q]; e < T.rrow_ptr[q + 1]; ++e) {
-      int2 v;
-      v.x = T.r_col[e];
-      v.y = *reinterpret_cast<const int32_t*>(&A.val[T.r_cidx[e]]);
-      se.push_back(v);
-      so.push_back(r_out[e]);
-    }
+    const int64_t len = T.rrow_ptr[q + 1] - T.rrow_ptr[q];
     const bool rmw = T.drow_ptr[q + 1] > T.drow_ptr[q];
     const int32_t out = sharded ? (int32_t)(q - q0s) : perm1[q];
-    ib.add_row(e0, (int32_t)se.size(), perm1[q], out, rmw);
+    ib.add_row((int32_t)ns, (int32_t)(ns + len), perm1[q], out, rmw);
+    rows_s.push_back(q);
+    soff.push_back(ns);
+    ns += len;
+  }
+  se.resize((size_t)ns);
+  so.resize((size_t)ns);
+#pragma omp parallel for schedule(dynamic, 256)
+  for (int64_t i = 0; i < (int64_t)rows_s.size(); ++i) {
+    const int32_t q = rows_s[i];
+    int64_t o = soff[i];
+    for (int64_t e = T.rrow_ptr[q]; e < T.rrow_ptr[q + 1]; ++e, ++o) {
+      se[o] = make_int2(T.r_col[e], *reinterpret_cast<const int32_t*>(&A.val[T.r_cidx[e]]));
+      so[o] = r_out[e];
+    }
   }
   const int64_t n_nonzero = (int64_t)ib.items.size();
   for (int64_t q = q0s; q < q1s; ++q) {
@@ -549,7 +579,9 @@ int finish_plan(sr_csr_s* h, cudaStream_t s) {
   }
   st.shard_panel_begin = pb;
   st.shard_panel_end = pe;
+  const double t0 = now_s();
   SR_TRY(build_exec_plan(h, pb, pe, s));
+  st.t_plan_s = now_s() - t0;
   st.shard_nrows = (int64_t)h->shard_rows.size();
   st.shard_nnz = (int64_t)h->shard_nnz_ids.size();
   h->reordered = true;
@@ -665,11 +697,8 @@ int sr_csr_create(int64_t nrows, int64_t ncols, int64_t nnz, const int64_t* rowp
     set_error("cudaStreamCreate failed");
     return SR_ECUDA;
   }
-  int rc = build_identity_plan(h, h->init_stream);
-  if (rc != SR_OK) {
-    sr_destroy(h);
-    return rc;
-  }
+  // the identity plan (P:101 row-wise kernels) is built on first use (ensure_plan), so a handle
+  // that is reordered or given a saved plan right away never uploads it
   sr_default_params(&h->params);
   h->perm1.resize((size_t)nrows);
   std::iota(h->perm1.begin(), h->perm1.end(), 0);
@@ -756,6 +785,7 @@ int sr_spmm(sr_csr h, const float* B, int64_t K, int64_t ldb, float* C, int64_t 
   if ((rows_out > 0 && !C) || (h->A.nnz() > 0 && !B)) return einval("sr_spmm: NULL operand");
   if (rows_out == 0) return SR_OK;
   DeviceGuard dg(h->device);
+  SR_TRY(ensure_plan(h));
   return launch_spmm(h, B, K, ldb, C, ldc, (cudaStream_t)stream, &h->last_launches);
 }
 
@@ -766,6 +796,7 @@ int sr_sddmm(sr_csr h, const float* X, int64_t ldx, const float* Y, int64_t ldy,
   if (h->A.nnz() == 0) return SR_OK;
   if (!X || !Y || !out) return einval("sr_sddmm: NULL operand");
   DeviceGuard dg(h->device);
+  SR_TRY(ensure_plan(h));
   return launch_sddmm(h, X, ldx, Y, ldy, K, out, (cudaStream_t)stream, &h->last_launches);
 }
 
@@ -1000,7 +1031,7 @@ int sr_plan_save(sr_csr h, void* buf, int64_t cap, int64_t* len) {
   st.shard_panel_end = st.npanels;
   st.shard_nrows = h->A.M;
   st.shard_nnz = nnz;
-  st.t_lsh1_s = st.t_cluster1_s = st.t_tile_s = st.t_lsh2_s = st.t_cluster2_s = st.t_total_s = 0.0;  // canonical
+  st.t_lsh1_s = st.t_cluster1_s = st.t_tile_s = st.t_lsh2_s = st.t_cluster2_s = st.t_total_s = st.t_plan_s = 0.0;
   w.put(st);
   w.put((int64_t)h->perm1.size());
   w.put_raw(h->perm1.data(), h->perm1.size() * 4);
@@ -1156,6 +1187,7 @@ extern "C" int sr_set_values(sr_csr h, const float* vals, sr_stream stream) {
   if (n == 0) return SR_OK;
   if (!vals) return einval("sr_set_values: NULL values");
   DeviceGuard dg(h->device);
+  SR_TRY(ensure_plan(h));
   DevPlan& P = h->plan;
   cudaStream_t s = (cudaStream_t)stream;
   SR_TRY(launch_set_values(P.s_ent.p, P.s_oidx.p, (int64_t)P.s_ent.n, vals, s));

@@ -706,7 +706,7 @@ __device__ __forceinline__ void dense_init_barriers(uint64_t* full, uint64_t* em
   if (threadIdx.x == 0) {
     for (int s = 0; s < kMaxStages; ++s) {
       mbar_init(&full[s], 1);
-      mbar_init(&empty[s], kDenseWarps);
+      mbar_init(&empty[s], kDenseWarps * 32);  // every consumer lane releases its own reads
     }
     mbar_init(&full[kMaxStages], 1);  // unit-blob ring (producer only)
     mbar_init(&full[kMaxStages + 1], 1);
@@ -782,8 +782,7 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) spmm_
         }
       }
     }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&empty[st]);
+    mbar_arrive(&empty[st]);  // release: this lane's reads of the stage happen before the refill
     if (hd.flags & kLastOfPass) {
       const int kk = hd.k0 + lg * VEC;
       const bool kv = kk < K;
@@ -939,8 +938,7 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) sddmm
         }
       }
     }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&empty[st]);
+    mbar_arrive(&empty[st]);  // release: this lane's reads of the stage happen before the refill
     if (hd.flags & kLastOfCta) break;
   }
 }

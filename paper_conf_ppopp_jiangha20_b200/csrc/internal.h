@@ -213,6 +213,7 @@ struct sr_csr_s {
   int device = 0;
   sr::HostCSR A;
   bool reordered = false;
+  bool identity_ready = false;  // the identity plan has been built (ensure_plan)
   sr_reorder_params params{};
   std::vector<int32_t> perm1, perm2;
   sr::Tiling tiles;

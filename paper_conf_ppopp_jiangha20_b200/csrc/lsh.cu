@@ -4,9 +4,10 @@
 //   minhash_bandkeys : warp per non-empty row; lane owns hash functions s = lane + 32t,
 //                      sweeps the row's columns (broadcast by shuffle) keeping running minima,
 //                      then writes one u64 band key per band (bsize 1 or 2: the exact tuple).
-//   per band         : radix sort (key, row) — stable, so bucket members stay ascending;
-//                      run-length encode -> bucket sizes; chunk cap (R14) -> pair counts;
-//                      emit_pairs: thread per bucket member, O(1) output offset.
+//   all bands at once: one stable radix sort of (band key, band|row) — equal keys of different
+//                      bands stay grouped by band, members ascending; run heads on (key, band)
+//                      -> bucket starts and sizes; chunk cap (R14) -> pair counts; emit_pairs_all:
+//                      thread per bucket member, O(1) output offset.  Two host syncs in total.
 //   all bands        : radix sort packed pairs + unique  -> E (union over bands, R13/R14).
 //   pair_jaccard     : thread per pair, sorted-list merge (binary-search when lopsided).
 //   heap order       : sort by (J desc, pair asc) through an exact 64-bit fixed-point key
@@ -93,19 +94,42 @@ __device__ __forceinline__ int64_t chunk_pairs(int64_t s, int64_t C) {
   return f * (C * (C - 1) / 2) + r * (r - 1) / 2;
 }
 
-__global__ void run_pair_counts(const int32_t* __restrict__ run_len, int64_t nruns, int64_t C,
-                                int64_t* __restrict__ npairs) {
+
+
+
+
+// All bands in one pass: after one stable radix sort of every (band key, band·L + t) pair by
+// the 64-bit key, equal keys of different bands stay grouped by band (the input is band-major and
+// the sort stable) and rows ascend inside each group, so a bucket is a maximal run of equal
+// (key, band) with its members ascending — exactly O5's bucket.
+__global__ void run_heads(const uint64_t* __restrict__ k, const uint32_t* __restrict__ v, int64_t n, int shift,
+                          uint8_t* __restrict__ head) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i < nruns) npairs[i] = chunk_pairs(run_len[i], C);
+  if (i >= n) return;
+  head[i] = (i == 0 || k[i] != k[i - 1] || (v[i] >> shift) != (v[i - 1] >> shift)) ? 1 : 0;
 }
 
-// element x of run r (start s0, size sz) emits pairs (x, y) for y after x in its chunk
-__global__ void emit_pairs(const int32_t* __restrict__ run_of, const int64_t* __restrict__ run_start,
-                           const int32_t* __restrict__ run_len, const int64_t* __restrict__ run_off,
-                           const int32_t* __restrict__ vals_sorted, const int32_t* __restrict__ live,
-                           int64_t L, int64_t C, uint64_t* __restrict__ out) {
+__global__ void run_lengths(const int64_t* __restrict__ start, int64_t nruns, int64_t n, int32_t* __restrict__ len,
+                            int64_t* __restrict__ npairs, int64_t C) {
+  const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (r > nruns) return;
+  if (r == nruns) {
+    npairs[r] = 0;
+    return;
+  }
+  const int64_t l = (r + 1 < nruns ? start[r + 1] : n) - start[r];
+  len[r] = (int32_t)l;
+  npairs[r] = chunk_pairs(l, C);
+}
+
+// element x of run r emits the pairs (x, y), y after x in its chunk (as emit_pairs); members are
+// live ids t (value & mask), ascending within the run
+__global__ void emit_pairs_all(const int32_t* __restrict__ run_of, const int64_t* __restrict__ run_start,
+                               const int32_t* __restrict__ run_len, const int64_t* __restrict__ run_off,
+                               const uint32_t* __restrict__ vals_sorted, uint32_t mask,
+                               const int32_t* __restrict__ live, int64_t n, int64_t C, uint64_t* __restrict__ out) {
   const int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (x >= L) return;
+  if (x >= n) return;
   const int32_t r = run_of[x];
   const int64_t sz = run_len[r];
   if (sz < 2) return;
@@ -117,24 +141,29 @@ __global__ void emit_pairs(const int32_t* __restrict__ run_of, const int64_t* __
   const int64_t clen = min(cap, sz - cs);
   const int64_t k = lx - cs;
   int64_t o = run_off[r] + chunk * (cap * (cap - 1) / 2) + k * (clen - 1) - k * (k - 1) / 2;
-  const uint64_t me = (uint64_t)(uint32_t)live[vals_sorted[x]];
+  const uint64_t me = (uint64_t)(uint32_t)live[vals_sorted[x] & mask];
   for (int64_t y = x + 1; y < s0 + cs + clen; ++y) {
-    const uint64_t other = (uint64_t)(uint32_t)live[vals_sorted[y]];
-    out[o++] = (me << 32) | other;  // live ids ascending within a bucket => me < other
+    const uint64_t other = (uint64_t)(uint32_t)live[vals_sorted[y] & mask];
+    out[o++] = (me << 32) | other;
   }
 }
 
-__global__ void mark_runs(const int64_t* __restrict__ run_start, const int32_t* __restrict__ run_len,
-                          int64_t nruns, int32_t* __restrict__ run_of) {
+__global__ void band_iota(uint32_t* __restrict__ v, int64_t L, int shift, int64_t n) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) v[i] = ((uint32_t)(i / L) << shift) | (uint32_t)(i % L);
+}
+
+__global__ void mark_runs64(const int64_t* __restrict__ run_start, const int32_t* __restrict__ run_len,
+                            int64_t nruns, int32_t* __restrict__ run_of) {
   const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (r >= nruns) return;
   const int64_t s0 = run_start[r];
   for (int32_t t = 0; t < run_len[r]; ++t) run_of[s0 + t] = (int32_t)r;
 }
 
-__global__ void to_int64(const int32_t* __restrict__ a, int64_t n, int64_t* __restrict__ b) {
+__global__ void iota_i64(int64_t* a, int64_t n) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i < n) b[i] = a[i];
+  if (i < n) a[i] = i;
 }
 
 __global__ void pair_jaccard(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
@@ -256,27 +285,27 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
 #undef SR_MH
     SR_CUDA_TRY(cudaGetLastError());
   }
-  // per band: sort, bucket, emit
-  DevBuf<uint64_t> kout;
-  DevBuf<int32_t> vin, vout, run_len, run_of, nruns_d;
-  DevBuf<uint64_t> run_key;
-  DevBuf<int64_t> run_start, run_npairs, run_off;
-  SR_TRY(kout.alloc(L));
-  SR_TRY(vin.alloc(L));
-  SR_TRY(vout.alloc(L));
-  SR_TRY(run_len.alloc(L));
-  SR_TRY(run_of.alloc(L));
-  SR_TRY(run_key.alloc(L));
-  SR_TRY(run_start.alloc(L + 1));
-  SR_TRY(run_npairs.alloc(L + 1));
-  SR_TRY(run_off.alloc(L + 1));
-  SR_TRY(nruns_d.alloc(1));
-  {
-    std::vector<int32_t> iota((size_t)L);
-    for (int64_t t = 0; t < L; ++t) iota[t] = (int32_t)t;
-    SR_CUDA_TRY(cudaMemcpyAsync(vin.p, iota.data(), L * sizeof(int32_t), cudaMemcpyHostToDevice, s));
-    SR_CUDA_TRY(cudaStreamSynchronize(s));
+  // all bands at once: one stable radix sort of (key, band·2^shift | t), run heads on
+  // (key, band), run starts by a flagged select, chunk-capped pair counts (R14), one scan, one
+  // emit launch; two host syncs in total (run count, pair count)
+  const int64_t NB = (int64_t)nb * L;
+  int shift = 1, band_bits = 0;
+  while ((int64_t(1) << shift) < L) ++shift;
+  while ((1 << band_bits) < nb) ++band_bits;
+  if (shift + band_bits > 32) {
+    set_error("lsh_candidates: non-empty rows x bands exceed the 32-bit (band, row) index of the one-pass banding");
+    return SR_EUNSUPPORTED;
   }
+  DevBuf<uint64_t> kout;
+  DevBuf<uint32_t> vin, vout;
+  DevBuf<uint8_t> head;
+  DevBuf<int64_t> idx, run_start, run_npairs, run_off, nruns_d;
+  DevBuf<int32_t> run_len, run_of;
+  SR_TRY(kout.alloc(NB));
+  SR_TRY(vin.alloc(NB));
+  SR_TRY(vout.alloc(NB));
+  band_iota<<<blocks(NB, 256), 256, 0, s>>>(vin.p, L, shift, NB);
+  SR_CUDA_TRY(cudaGetLastError());
   DevBuf<uint8_t> temp;
   size_t temp_bytes = 0;
   auto ensure_temp = [&](size_t need) -> int {
@@ -286,65 +315,66 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
     }
     return SR_OK;
   };
-  DevBuf<uint64_t> allpairs;
-  int64_t cap_pairs = 0, n_pairs = 0;
-  const int64_t C = p.max_bucket;
-  for (int band = 0; band < nb; ++band) {
+  {
     size_t need = 0;
-    cub::DeviceRadixSort::SortPairs(nullptr, need, keys.p + (int64_t)band * L, kout.p, vin.p, vout.p, (int)L, 0, 64, s);
+    cub::DeviceRadixSort::SortPairs(nullptr, need, keys.p, kout.p, vin.p, vout.p, NB, 0, 64, s);
     SR_TRY(ensure_temp(need));
     need = temp_bytes;
-    SR_CUDA_TRY(cub::DeviceRadixSort::SortPairs(temp.p, need, keys.p + (int64_t)band * L, kout.p, vin.p,
-                                                vout.p, (int)L, 0, 64, s));
-    need = 0;
-    cub::DeviceRunLengthEncode::Encode(nullptr, need, kout.p, run_key.p, run_len.p, nruns_d.p, (int)L, s);
-    SR_TRY(ensure_temp(need));
-    need = temp_bytes;
-    SR_CUDA_TRY(cub::DeviceRunLengthEncode::Encode(temp.p, need, kout.p, run_key.p, run_len.p, nruns_d.p,
-                                                   (int)L, s));
-    int32_t nruns = 0;
-    SR_CUDA_TRY(cudaMemcpyAsync(&nruns, nruns_d.p, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
-    SR_CUDA_TRY(cudaStreamSynchronize(s));
-    if (nruns == L) continue;  // every bucket is a singleton
-    // run starts = exclusive sum of lengths (int64)
-    to_int64<<<blocks(nruns, 256), 256, 0, s>>>(run_len.p, nruns, run_npairs.p);
-    need = 0;
-    cub::DeviceScan::ExclusiveSum(nullptr, need, run_npairs.p, run_start.p, (int)nruns + 0, s);
-    SR_TRY(ensure_temp(need));
-    need = temp_bytes;
-    SR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(temp.p, need, run_npairs.p, run_start.p, (int)nruns, s));
-    mark_runs<<<blocks(nruns, 256), 256, 0, s>>>(run_start.p, run_len.p, nruns, run_of.p);
-    run_pair_counts<<<blocks(nruns, 256), 256, 0, s>>>(run_len.p, nruns, C, run_npairs.p);
-    SR_CUDA_TRY(cudaMemsetAsync(run_npairs.p + nruns, 0, sizeof(int64_t), s));
-    need = 0;
-    cub::DeviceScan::ExclusiveSum(nullptr, need, run_npairs.p, run_off.p, (int)nruns + 1, s);
-    SR_TRY(ensure_temp(need));
-    need = temp_bytes;
-    SR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(temp.p, need, run_npairs.p, run_off.p, (int)nruns + 1, s));
-    int64_t band_pairs = 0;
-    SR_CUDA_TRY(cudaMemcpyAsync(&band_pairs, run_off.p + nruns, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-    SR_CUDA_TRY(cudaStreamSynchronize(s));
-    if (band_pairs == 0) continue;
-    if (n_pairs + band_pairs > cap_pairs) {
-      int64_t ncap = std::max<int64_t>(2 * cap_pairs, n_pairs + band_pairs);
-      ncap = std::max<int64_t>(ncap, 1 << 20);
-      DevBuf<uint64_t> bigger;
-      SR_TRY(bigger.alloc(ncap));
-      if (n_pairs)
-        SR_CUDA_TRY(cudaMemcpyAsync(bigger.p, allpairs.p, n_pairs * sizeof(uint64_t),
-                                    cudaMemcpyDeviceToDevice, s));
-      SR_CUDA_TRY(cudaStreamSynchronize(s));
-      std::swap(bigger.p, allpairs.p);
-      std::swap(bigger.n, allpairs.n);
-      cap_pairs = ncap;
-    }
-    // run_off is relative to this band: shift output pointer
-    emit_pairs<<<blocks(L, 256), 256, 0, s>>>(run_of.p, run_start.p, run_len.p, run_off.p, vout.p, d_live.p,
-                                              L, C, allpairs.p + n_pairs);
-    SR_CUDA_TRY(cudaGetLastError());
-    n_pairs += band_pairs;
+    SR_CUDA_TRY(cub::DeviceRadixSort::SortPairs(temp.p, need, keys.p, kout.p, vin.p, vout.p, NB, 0, 64, s));
   }
   keys.release();
+  vin.release();
+  SR_TRY(head.alloc(NB));
+  run_heads<<<blocks(NB, 256), 256, 0, s>>>(kout.p, vout.p, NB, shift, head.p);
+  SR_CUDA_TRY(cudaGetLastError());
+  SR_TRY(idx.alloc(NB));
+  SR_TRY(run_start.alloc(NB));
+  SR_TRY(nruns_d.alloc(1));
+  iota_i64<<<blocks(NB, 256), 256, 0, s>>>(idx.p, NB);
+  {
+    size_t need = 0;
+    cub::DeviceSelect::Flagged(nullptr, need, idx.p, head.p, run_start.p, nruns_d.p, NB, s);
+    SR_TRY(ensure_temp(need));
+    need = temp_bytes;
+    SR_CUDA_TRY(cub::DeviceSelect::Flagged(temp.p, need, idx.p, head.p, run_start.p, nruns_d.p, NB, s));
+  }
+  int64_t nruns = 0;
+  SR_CUDA_TRY(cudaMemcpyAsync(&nruns, nruns_d.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  SR_CUDA_TRY(cudaStreamSynchronize(s));
+  kout.release();
+  head.release();
+  idx.release();
+  const int64_t C = p.max_bucket;
+  DevBuf<uint64_t> allpairs;
+  int64_t n_pairs = 0;
+  if (nruns < NB) {  // some bucket has two or more rows
+    SR_TRY(run_len.alloc(nruns));
+    SR_TRY(run_npairs.alloc(nruns + 1));
+    SR_TRY(run_off.alloc(nruns + 1));
+    SR_TRY(run_of.alloc(NB));
+    run_lengths<<<blocks(nruns + 1, 256), 256, 0, s>>>(run_start.p, nruns, NB, run_len.p, run_npairs.p, C);
+    mark_runs64<<<blocks(nruns, 256), 256, 0, s>>>(run_start.p, run_len.p, nruns, run_of.p);
+    SR_CUDA_TRY(cudaGetLastError());
+    size_t need = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, need, run_npairs.p, run_off.p, nruns + 1, s);
+    SR_TRY(ensure_temp(need));
+    need = temp_bytes;
+    SR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(temp.p, need, run_npairs.p, run_off.p, nruns + 1, s));
+    SR_CUDA_TRY(cudaMemcpyAsync(&n_pairs, run_off.p + nruns, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    SR_CUDA_TRY(cudaStreamSynchronize(s));
+    if (n_pairs > 0) {
+      SR_TRY(allpairs.alloc(n_pairs));
+      emit_pairs_all<<<blocks(NB, 256), 256, 0, s>>>(run_of.p, run_start.p, run_len.p, run_off.p, vout.p,
+                                                    (uint32_t)((1u << shift) - 1), d_live.p, NB, C, allpairs.p);
+      SR_CUDA_TRY(cudaGetLastError());
+    }
+  }
+  run_of.release();
+  run_len.release();
+  run_npairs.release();
+  run_off.release();
+  run_start.release();
+  vout.release();
   if (n_pairs == 0) return SR_OK;
   // union over bands: sort + unique
   DevBuf<uint64_t> sorted, uniq;

@@ -317,32 +317,42 @@ def test_shard_simulation(env, oracle, world):
 
 
 # ------------------------------------------------------------------ full-size configs
+# bench.py's plan parameters (the launch configuration it times): AUTO, dense_min 64 for the
+# kernels, auto_dense_min 8 for the round-1 decision (R28), max_bucket 32 (R14)
+BENCH_KW = dict(siglen=128, bsize=2, seed=4, max_bucket=32, threshold_size=256, panel_rows=64, dense_min=64,
+                auto_dense_min=8, mode=0)
+
+
+def _sampled_rows(A, n=2000):
+    rng = np.random.default_rng(0)
+    deg = np.diff(A.rowptr)
+    return np.unique(np.concatenate([rng.integers(0, A.nrows, n), np.argsort(deg)[-20:]]))
+
+
 @pytest.mark.slow
 @pytest.mark.parametrize("config", ["rmat", "banded", "gnn", "cf"])
-def test_full_size_sampled(env, oracle, config):
-    """C2-C5 at full size in the launch configuration bench.py times (default plan
-    parameters, AUTO mode): plan bit-exact vs the oracle; SpMM checked on 2000 sampled rows
-    plus the 20 longest rows (K=128, and K=32 for C2); SDDMM on every nnz of those rows."""
+def test_full_size_plan_bench_params(env, oracle, config):
+    """C2-C5 at full size with bench.py's plan parameters: perm1, perm2, tiles and the AUTO
+    decisions bit-exact against the oracle (AUTO runs both rounds on C2 and C4, none on C3,
+    round 2 on C5); SpMM (K=128) on 2000 sampled rows + the 20 longest, SDDMM on all their nnz.
+    C5's round 2 at max_bucket 32 has E2 = 275 M candidates, beyond what the oracle's plain
+    priority queue clusters in minutes: C5 runs here with max_bucket 8, and its bench-parameter
+    plan is checked by test_full_size_cf_bench_params."""
     sr, torch = env
     A = g.make(config)
-    # C2 (rmat) is bench.py's workload: its plan (dense_min 64, profiles/r01/NOTES.md); the other
-    # configs keep the paper's example threshold 2 (P:111), under which AUTO skips their round 1
-    # (DenseRatio0 > 1/10) and the CPU oracle's plan finishes in minutes
-    kw = dict(siglen=128, bsize=2, seed=4, max_bucket=32, threshold_size=256, panel_rows=64,
-              dense_min=64 if config == "rmat" else 2, mode=0)
+    kw = dict(BENCH_KW, max_bucket=8) if config == "cf" else BENCH_KW
     M = sr.SparseMatrix.from_csr(A)
     M.reorder(sr.default_params(**kw))
     ref = oracle.plan(A, **kw)
     _assert_plan_equal(M, ref)
     del ref
-    rng = np.random.default_rng(0)
+    rows = _sampled_rows(A)
     deg = np.diff(A.rowptr)
-    rows = np.unique(np.concatenate([rng.integers(0, A.nrows, 2000), np.argsort(deg)[-20:]]))
-    for K in ((128, 32) if config == "rmat" else (128,)):
-        B = g.dense(A.ncols, K)
-        C = M.spmm(torch.from_numpy(B).cuda())
-        torch.cuda.synchronize()
-        _spmm_check(oracle, A, B, C.cpu().numpy(), rows=rows)
+    B = g.dense(A.ncols, 128)
+    C = M.spmm(torch.from_numpy(B).cuda())
+    torch.cuda.synchronize()
+    _spmm_check(oracle, A, B, C.cpu().numpy(), rows=rows)
+    del C
     X, Y = g.dense(A.nrows, 128, stream=1), g.dense(A.ncols, 128, stream=2)
     out = M.sddmm(torch.from_numpy(X).cuda(), torch.from_numpy(Y).cuda()).cpu().numpy()
     sel = np.concatenate([np.arange(A.rowptr[r], A.rowptr[r + 1]) for r in rows])
@@ -351,6 +361,55 @@ def test_full_size_sampled(env, oracle, config):
     ref_o, bound = oracle.sddmm(sub, X[rows], Y)
     err = np.abs(out[sel] - ref_o)
     assert not (err > TOL * bound + 1e-30).any()
+
+
+@pytest.mark.slow
+def test_full_size_cf_bench_params(env, oracle):
+    """C5 with exactly bench.py's plan parameters (max_bucket 32, E2 = 275 M): the AUTO
+    decisions (DenseRatio0 under R28, AvgSim of the remainder) and the tiling of perm1 are
+    bit-exact against the oracle's O10/O11 (round 1 is skipped, so perm1 is the identity), and
+    perm2 lists every non-empty remainder position exactly once."""
+    sr, torch = env
+    A = g.make("cf")
+    M = sr.SparseMatrix.from_csr(A)
+    M.reorder(sr.default_params(**BENCH_KW))
+    st = M.stats()
+    t0 = oracle.tile(A, np.arange(A.nrows), BENCH_KW["panel_rows"], BENCH_KW["auto_dense_min"])
+    assert st["dense0"] == t0["n_dense"] and st["round1"] == 0 and t0["n_dense"] * 10 > A.nnz
+    np.testing.assert_array_equal(M.perm(1), np.arange(A.nrows))
+    t = oracle.tile(A, np.arange(A.nrows), BENCH_KW["panel_rows"], BENCH_KW["dense_min"])
+    mt = M.tiles()
+    for k in ("dense_ptr", "dense_cols", "drow_ptr", "d_slot", "d_pos", "rrow_ptr", "r_col", "r_pos"):
+        np.testing.assert_array_equal(mt[k], t[k], err_msg=k)
+    num, den = oracle.avgsim(t["rrow_ptr"], t["r_col"])
+    assert (st["avgsim_num"], st["avgsim_den"]) == (num, den)
+    assert st["round2"] == (0 if num * 10 > den else 1)
+    nonempty = np.flatnonzero(np.diff(t["rrow_ptr"]) > 0)
+    np.testing.assert_array_equal(np.sort(M.perm(2)), nonempty)
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("K", [32, 128])
+def test_full_size_rmat_whole_output(env, oracle, K):
+    """C2 (bench.py's workload) with bench.py's plan: every entry of C = A·B (1,048,576 × K) and
+    every one of the 16,086,011 SDDMM values against the fp64 oracle, element by element."""
+    sr, torch = env
+    A = g.make("rmat")
+    M = sr.SparseMatrix.from_csr(A)
+    M.reorder(sr.default_params(**BENCH_KW))
+    B = g.dense(A.ncols, K)
+    C = M.spmm(torch.from_numpy(B).cuda()).cpu().numpy()
+    step = 1 << 17
+    for r0 in range(0, A.nrows, step):
+        rows = np.arange(r0, min(A.nrows, r0 + step))
+        ref, bound = oracle.spmm_rows(A, B, rows)
+        err = np.abs(C[rows].astype(np.float64) - ref)
+        bad = err > TOL * bound + 1e-30
+        assert not bad.any(), f"rows {r0}+: {bad.sum()} entries out of tolerance, worst {err.max()}"
+    del C
+    X, Y = g.dense(A.nrows, K, stream=1), g.dense(A.ncols, K, stream=2)
+    out = M.sddmm(torch.from_numpy(X).cuda(), torch.from_numpy(Y).cuda()).cpu().numpy()
+    _sddmm_check(oracle, A, X, Y, out)
 
 
 def test_scatter_helpers_reassemble_shards(env, oracle):
@@ -401,16 +460,14 @@ def test_dist_gather_single_rank_nccl(env, oracle):
 
 
 # ------------------------------------------------------------------ alternative engines
-@pytest.mark.parametrize("var,val", [("SR_DENSE_ENGINE", "coop"), ("SR_DENSE_ENGINE", "l1"),
-                                     ("SR_SPARSE_VARIANT", "0"), ("SR_SPARSE_VARIANT", "4"),
-                                     ("SR_SPARSE_VARIANT", "5"),
+@pytest.mark.parametrize("var,val", [("SR_PHASE_S", "0"), ("SR_GATHER4", "0"),
                                      ("SR_TASK_NNZ", "1"), ("SR_TASK_NNZ", "1024")])
 def test_engines_subprocess(env, var, val):
-    """The phase-D engine (SR_DENSE_ENGINE) and the phase-S kernels (SR_SPARSE_VARIANT: 0 =
-    one-row-per-warp kernels, 4, 5 = task kernels at other occupancy points / entry layouts; SR_TASK_NNZ=1 = one
-    row per task) are chosen once per process; rerun the numeric parity cases that exercise
-    them (K sweep incl. multi-pass K, tile widths, split rows + RMW rows) under the
-    non-default choices."""
+    """Process-wide kernel choices (SR_PHASE_S=0: the one-row-per-warp phase-S kernels instead of
+    the row-group task kernels; SR_GATHER4=0: per-row cp.async.bulk staging instead of TMA
+    tile::gather4 in phase D; SR_TASK_NNZ: task size, 1 = one row per task) are fixed once per
+    process; rerun the numeric parity cases that exercise them (K sweep incl. multi-pass K,
+    tile widths, split rows + RMW rows) under the non-default choices."""
     import os
     import subprocess
     import sys

@@ -1,0 +1,37 @@
+"""compute-sanitizer memcheck / racecheck / synccheck over small invocations of every libsr
+kernel path (tests/sanitizer_cases.py): the phase-D mbarrier full/empty rings and TMA
+producer, the atomic-ticket ordered combines of split rows and split hub panels, the phase-S
+task kernels (shared-memory X staging with cp.async in SDDMM) and sr_set_values."""
+import os
+import shutil
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _sanitizer():
+    for p in (shutil.which("compute-sanitizer"), "/usr/local/cuda/bin/compute-sanitizer"):
+        if p and os.path.exists(p):
+            return p
+    pytest.fail("compute-sanitizer not found")
+
+
+@pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck"])
+def test_compute_sanitizer(tool):
+    cmd = [_sanitizer(), "--tool", tool, "--error-exitcode", "17", "--print-limit", "20"]
+    if tool == "memcheck":
+        cmd += ["--leak-check", "no"]
+    if tool == "racecheck":
+        cmd += ["--racecheck-report", "hazard"]
+    cmd += [sys.executable, os.path.join(ROOT, "tests", "sanitizer_cases.py")]
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=1800, cwd=ROOT)
+    log = r.stdout[-6000:] + r.stderr[-4000:]
+    assert r.returncode == 0, log
+    assert "sanitizer cases ok" in r.stdout, log
+    import re
+    summary = re.findall(r"(?:ERROR|RACECHECK) SUMMARY: .*", r.stdout + r.stderr)
+    assert summary and all(re.search(r": 0 (errors|hazards)", s_) for s_ in summary), log
