@@ -304,6 +304,10 @@ def algorithmic_bytes(kind: str, tm: dict, K: int) -> float:
     if kind == "spmm_sparse_rows":
         return (8.0 * tm["sparse_nnz"] + 16.0 * tm["sparse_items"] + row * tm["sparse_distinct_cols"]
                 + row * (tm["sparse_rows"] + tm["zero_rows"]) + row * tm["rmw_rows"])
+    if kind == "spmm_register_tiles":  # the dense part on the register-tile engine
+        kind = "spmm_dense_tiles"
+    if kind == "sddmm_register_tiles":
+        kind = "sddmm_dense_tiles"
     if kind == "spmm_dense_tiles":
         return 8.0 * tm["dense_nnz"] + row * tm["dense_distinct_cols"] + row * tm["dense_rows"]
     if kind == "sddmm_sparse_rows":

@@ -268,7 +268,8 @@ int sr_get_traffic_model(sr_csr h, sr_traffic_model* out);
 int sr_set_profiling(sr_csr h, int enable);
 
 /* Device time of each launch of the last sr_spmm / sr_sddmm call (waits for its events).
- * kinds: 1 = spmm phase D, 2 = spmm phase S, 3 = sddmm phase D, 4 = sddmm phase S. */
+ * kinds: 1 = spmm phase D (TMA shared-memory tiles), 2 = spmm phase S, 3 = sddmm phase D (TMA),
+ *        4 = sddmm phase S, 5 = spmm phase D on register tiles, 6 = sddmm phase D on register tiles. */
 int sr_last_kernel_times(sr_csr h, int32_t* kinds, float* ms, int32_t cap, int32_t* n);
 
 const char* sr_last_error(void);

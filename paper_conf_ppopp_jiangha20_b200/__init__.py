@@ -64,7 +64,8 @@ class TrafficModel(C.Structure):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
 
-KERNEL_KINDS = {1: "spmm_dense_tiles", 2: "spmm_sparse_rows", 3: "sddmm_dense_tiles", 4: "sddmm_sparse_rows"}
+KERNEL_KINDS = {1: "spmm_dense_tiles", 2: "spmm_sparse_rows", 3: "sddmm_dense_tiles", 4: "sddmm_sparse_rows",
+                5: "spmm_register_tiles", 6: "sddmm_register_tiles"}
 
 EXPORTED = ("sr_csr_create", "sr_default_params", "sr_reorder", "sr_spmm", "sr_sddmm", "sr_destroy",
             "sr_get_perm", "sr_get_plan_stats", "sr_export_tiles", "sr_shard_rows", "sr_shard_nnz_ids",

@@ -1,6 +1,7 @@
 // C ABI of libsr (include/sr.h): ingest, the reorder driver (Fig 5 workflow, P:137;
 // decision rules P:265), plan construction, metadata export, host entry points.
 #include <algorithm>
+#include <array>
 #include <chrono>
 #include <cstdlib>
 #include <cstring>
@@ -218,6 +219,65 @@ int build_identity_plan(sr_csr_s* h, cudaStream_t s) {
   return SR_OK;
 }
 
+// Register-tile stream of the dense nnz (panels of <= kRtMaxRows rows, exec.cu:
+// spmm_rtile_kernel / sddmm_rtile_kernel).  Per panel, its dense columns in slot order (count
+// desc, column asc: R18); per column one header entry {col | kRtHeader, mask of the panel rows
+// holding it} followed by one {row, value bits} entry per such row, rows ascending.  A column's
+// entries never straddle a 32-entry batch of its panel (padding entries {0, 0} in between), so
+// a warp decodes each batch on its own.  Units (one warp per panel) are ordered largest first.
+int build_rt_stream(sr_csr_s* h, int64_t pb, int64_t pe, const std::vector<int32_t>& d_out, DevPlan& P,
+                    cudaStream_t s) {
+  const HostCSR& A = h->A;
+  const Tiling& T = h->tiles;
+  const int64_t M = A.M;
+  const int32_t PR = h->params.panel_rows;
+  std::vector<int2> ent;
+  std::vector<int32_t> oidx;
+  std::vector<int4> units;
+  std::vector<std::array<int32_t, 3>> cell;  // (slot, row, dense nnz index)
+  for (int64_t p = pb; p < pe; ++p) {
+    const int64_t dc0 = T.dense_ptr[p], dc1 = T.dense_ptr[p + 1];
+    if (dc1 == dc0) continue;
+    const int64_t q0 = p * PR, nrows = std::min<int64_t>(M, q0 + PR) - q0;
+    if (T.drow_ptr[q0 + nrows] - T.drow_ptr[q0] > kRtMaxPanelEntries) continue;  // TMA engine
+    cell.clear();
+    for (int64_t r = 0; r < nrows; ++r)
+      for (int64_t e = T.drow_ptr[q0 + r]; e < T.drow_ptr[q0 + r + 1]; ++e)
+        cell.push_back({T.d_slot[e], (int32_t)r, (int32_t)e});
+    std::sort(cell.begin(), cell.end());
+    const int64_t e0 = (int64_t)ent.size();
+    size_t i = 0;
+    while (i < cell.size()) {
+      size_t j = i;
+      uint32_t mask = 0;
+      while (j < cell.size() && cell[j][0] == cell[i][0]) mask |= 1u << cell[j++][1];
+      const int64_t len = 1 + (int64_t)(j - i), at = ((int64_t)ent.size() - e0) % 32;
+      if (at + len > 32)  // keep the column inside one 32-entry batch
+        for (int64_t k = at; k < 32; ++k) {
+          ent.push_back(make_int2(0, 0));
+          oidx.push_back(-1);
+        }
+      ent.push_back(make_int2((int32_t)(T.dense_cols[dc0 + cell[i][0]] | kRtHeader), (int32_t)mask));
+      oidx.push_back(-1);
+      for (size_t k = i; k < j; ++k) {
+        const int64_t e = cell[k][2];
+        ent.push_back(make_int2(cell[k][1], *reinterpret_cast<const int32_t*>(&A.val[T.d_cidx[e]])));
+        oidx.push_back(d_out[e]);
+      }
+      i = j;
+    }
+    units.push_back(make_int4((int32_t)e0, (int32_t)ent.size(), (int32_t)q0, (int32_t)nrows));
+  }
+  std::stable_sort(units.begin(), units.end(), [](const int4& a, const int4& b) { return a.y - a.x > b.y - b.x; });
+  ent.resize(ent.size() + kEntPad, make_int2(0, 0));
+  oidx.resize(oidx.size() + kEntPad, -1);
+  P.n_rt = (int64_t)units.size();
+  SR_TRY(P.rt_units.upload(units, s));
+  SR_TRY(P.rt_ent.upload(ent, s));
+  SR_TRY(P.rt_oidx.upload(oidx, s));
+  return SR_OK;
+}
+
 // The identity plan on first use of a handle without a reordered plan.  Synchronous (once).
 int ensure_plan(sr_csr_s* h) {
   if (h->reordered || h->identity_ready) return SR_OK;
@@ -318,10 +378,15 @@ int build_exec_plan_into(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s, De
       deo.push_back(-1);
     }
   };
+  // panels of <= kRtMaxRows rows run on the register-tile engine (build_rt_stream) instead
+  // except panels with more than kRtMaxPanelEntries dense nnz (hub rows: one warp would serialise
+  // them), which stay on this engine with its split units and ordered combine
+  const bool rt = PR <= kRtMaxRows;
   for (int64_t p = pb; p < pe; ++p) {
     const int64_t dc0 = T.dense_ptr[p], dc1 = T.dense_ptr[p + 1];
     if (dc1 == dc0) continue;
     const int64_t q0 = p * PR, nrows = std::min<int64_t>(M, q0 + PR) - q0;
+    if (rt && T.drow_ptr[q0 + nrows] - T.drow_ptr[q0] <= kRtMaxPanelEntries) continue;
     const int64_t nd = dc1 - dc0, nt = (nd + TW - 1) / TW;
     maxd = std::max(maxd, nd);
     for (int64_t r = 0; r < nrows; ++r) cur[r] = T.drow_ptr[q0 + r];
@@ -380,6 +445,7 @@ int build_exec_plan_into(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s, De
     if (nunits > 1) n_dslots += nunits;
   }
   pad4();
+  if (rt) SR_TRY(build_rt_stream(h, pb, pe, d_out, P, s));
   P.n_units = (int64_t)units.size();
   P.max_dense_per_panel = maxd;
   P.tile_cols = TW;
@@ -482,7 +548,20 @@ int build_exec_plan_into(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s, De
           ++tm.dense_distinct_cols;
         }
     }
-    tm.dense_panels = (int64_t)units.size();
+    if (rt) {  // register tiles: every dense column of a panel is gathered once per K pass
+      for (int64_t p = pb; p < pe; ++p) {
+        const int64_t q0 = p * PR, q1 = std::min<int64_t>(M, q0 + PR);
+        if (T.drow_ptr[q1] - T.drow_ptr[q0] > kRtMaxPanelEntries) continue;  // counted with the vtiles
+        for (int64_t k = T.dense_ptr[p]; k < T.dense_ptr[p + 1]; ++k) {
+          ++tm.dense_col_loads;
+          if (!seen[T.dense_cols[k]]) {
+            seen[T.dense_cols[k]] = 1;
+            ++tm.dense_distinct_cols;
+          }
+        }
+      }
+    }
+    tm.dense_panels = P.n_rt + (int64_t)units.size();
     for (int64_t q = q0s; q < q1s; ++q) {
       const bool d = T.drow_ptr[q + 1] > T.drow_ptr[q], r = T.rrow_ptr[q + 1] > T.rrow_ptr[q];
       tm.dense_nnz += T.drow_ptr[q + 1] - T.drow_ptr[q];
@@ -1192,5 +1271,6 @@ extern "C" int sr_set_values(sr_csr h, const float* vals, sr_stream stream) {
   cudaStream_t s = (cudaStream_t)stream;
   SR_TRY(launch_set_values(P.s_ent.p, P.s_oidx.p, (int64_t)P.s_ent.n, vals, s));
   if (P.n_units > 0) SR_TRY(launch_set_values(P.d_ent.p, P.d_oidx.p, (int64_t)P.d_ent.n, vals, s));
+  if (P.n_rt > 0) SR_TRY(launch_set_values(P.rt_ent.p, P.rt_oidx.p, (int64_t)P.rt_ent.n, vals, s));
   return SR_OK;
 }

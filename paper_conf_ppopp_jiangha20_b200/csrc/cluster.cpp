@@ -119,6 +119,11 @@ class PairSet {
     }
   }
   void set_size(size_t n) { size_ = n; }
+  size_t size() const { return size_; }
+  // make room for `more` insertions without growing inside a parallel region
+  void reserve_more(size_t more) {
+    while (2 * (size_ + more + 1) > cap_) grow();
+  }
   void insert(uint64_t k) {
     if (2 * (size_ + 1) > cap_) grow();
     size_t h = hash(k) & mask_;
@@ -158,6 +163,47 @@ class PairSet {
   }
   std::unique_ptr<uint64_t[]> slots_;
   size_t cap_ = 0, mask_ = 0, size_ = 0;
+};
+
+// Keys inserted since the last flush into the big membership set (L2-resident, cleared through
+// its list of used slots).
+class SmallSet {
+ public:
+  SmallSet() : slots_(kCap, kEmpty) {}
+  bool contains(uint64_t k) const {
+    size_t h = mix(k);
+    while (true) {
+      const uint64_t v = slots_[h];
+      if (v == k) return true;
+      if (v == kEmpty) return false;
+      h = (h + 1) & (kCap - 1);
+    }
+  }
+  void insert(uint64_t k) {
+    size_t h = mix(k);
+    while (slots_[h] != kEmpty) {
+      if (slots_[h] == k) return;
+      h = (h + 1) & (kCap - 1);
+    }
+    slots_[h] = k;
+    used_.push_back((uint32_t)h);
+    keys_.push_back(k);
+  }
+  bool nearly_full() const { return used_.size() * 2 > kCap; }
+  const std::vector<uint64_t>& keys() const { return keys_; }
+  void clear() {
+    for (uint32_t h : used_) slots_[h] = kEmpty;
+    used_.clear();
+    keys_.clear();
+  }
+
+ private:
+  static constexpr size_t kCap = 1 << 14;
+  static constexpr uint64_t kEmpty = ~0ull;
+  static size_t mix(uint64_t k) { return (size_t)((k * 0x9E3779B97F4A7C15ull) >> 50) & (kCap - 1); }
+  std::vector<uint64_t> slots_;
+  std::vector<uint32_t> used_;
+  std::vector<uint64_t> keys_;
 };
 
 inline void intersect(const int64_t* rowptr, const int32_t* col, int64_t a, int64_t b,
@@ -233,12 +279,24 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
     for (int64_t r = 0; r <= M; ++r)
       seg[r] = std::lower_bound(pairs_by_key, pairs_by_key + npairs, (uint64_t)r << 32) - pairs_by_key;
   }
-  auto is_candidate = [&](uint64_t key) {
+  SmallSet recent;  // re-inserted pairs not yet flushed into `members` (see flush_recent)
+  auto is_candidate_big = [&](uint64_t key) {
     if (by_key) {
       const int64_t lo = (int64_t)(key >> 32);
       if (std::binary_search(pairs_by_key + seg[lo], pairs_by_key + seg[lo + 1], key)) return true;
     }
     return members.contains(key);
+  };
+  auto is_candidate = [&](uint64_t key) { return recent.contains(key) || is_candidate_big(key); };
+  // move the recent re-inserts into the big set (distinct keys, absent from it: parallel CAS)
+  auto flush_recent = [&]() {
+    const std::vector<uint64_t>& ks = recent.keys();
+    if (ks.empty()) return;
+    members.reserve_more(ks.size());
+#pragma omp parallel for schedule(static) if (ks.size() > 4096)
+    for (int64_t k = 0; k < (int64_t)ks.size(); ++k) members.insert_distinct_concurrent(ks[k]);
+    members.set_size(members.size() + ks.size());
+    recent.clear();
   };
   const double ta = now();
   std::vector<RowDigest> dig((size_t)M);
@@ -316,11 +374,154 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
   while (init_pos > 0 && init[init_pos - 1].inter == 0) --init_pos;
   size_t cur = 0, zc = 0;
   int64_t nclusters = M;
-  constexpr size_t PF = 32, PF2 = 16, PF3 = 8;  // prefetch distances over the initial-candidate cursor
+  // roots changed by a merge since the current block's speculative evaluation: a 4096-bit
+  // filter (false positives only send a pop down the sequential path)
+  uint64_t modbits[64];
+  auto mod_bit = [](int32_t x) { return (uint32_t)((uint32_t)x * 0x9E3779B1u) >> 20; };
+  auto mark_mod = [&](int32_t x) { const uint32_t b = mod_bit(x); modbits[b >> 6] |= 1ull << (b & 63); };
+  auto is_mod = [&](int32_t x) { const uint32_t b = mod_bit(x); return (modbits[b >> 6] >> (b & 63)) & 1ull; };
+  std::memset(modbits, 0, sizeof(modbits));
+  bool midflush = false;  // `recent` was flushed since the current block's evaluation
+  auto reinsert = [&](const Cand& c, uint64_t key) {
+    if (recent.nearly_full()) {
+      flush_recent();
+      midflush = true;
+    }
+    recent.insert(key);
+    ++n_reinsert;
+    if (c.inter > 0) {
+      extra.push(c);
+    } else {
+      ++n_zero;
+      if (zero_phase)
+        zero_new.push(key);
+      else
+        zero_keys.push_back(key);
+    }
+  };
+  // One popped pair, exactly as Alg 3 (lines 17-30 under R3-R12): the sequential path.
+  auto process = [&](int32_t i, int32_t j) {
+    if (nd[i].parent == i && nd[j].parent == j) {
+      if ((nd[i].sz | nd[j].sz) & kDeleted) return;
+      // the larger cluster absorbs the smaller; equal sizes: smaller index (R6)
+      const bool i_wins = nd[i].sz > nd[j].sz || (nd[i].sz == nd[j].sz && i < j);
+      const int32_t w = i_wins ? i : j, l = i_wins ? j : i;
+      nd[l].parent = w;
+      nd[w].sz += nd[l].sz;  // R4
+      --nclusters;
+      if (nd[w].sz >= (uint32_t)threshold_size) {  // R7, R5
+        nd[w].sz |= kDeleted;
+        --nclusters;
+      }
+      mark_mod(w);
+      mark_mod(l);
+    } else {
+      i = root(i);
+      j = root(j);
+      if (((nd[i].sz | nd[j].sz) & kDeleted) || i == j) return;
+      const uint32_t lo = (uint32_t)std::min(i, j), hi = (uint32_t)std::max(i, j);
+      const uint64_t key = ((uint64_t)lo << 32) | hi;
+      if (is_candidate(key)) return;
+      Cand c;
+      similarity(lo, hi, &c);  // representing rows (R8)
+      reinsert(c, key);
+    }
+  };
+  // Speculative evaluation of the initial-candidate cursor in blocks (parallel, read-only):
+  // against the union-find state at the block's start, each pop is classified as
+  //   0 both rows are roots -> merge path, done sequentially at its turn;
+  //   1 the roots are equal or one is deleted -> skip (both facts are permanent: a deleted root
+  //     never merges again and equal roots stay equal), valid whatever happens in between;
+  //   2 the roots' pair is a candidate -> skip, valid if neither root changed since;
+  //   3 not a candidate -> re-insert with the exact J computed here (the expensive part), valid
+  //     if neither root changed since and no earlier pop of the block re-inserted the same pair.
+  // The pops then run in the exact sequential order (interleaved with the re-insert heap); a
+  // pop whose class 2/3 result may be stale (a root merged since, modbits) takes the
+  // sequential path.  The result is identical to the plain loop.
+  const bool spec = getenv("SR_CLUSTER_SEQ") == nullptr;
+  struct Pre {
+    int32_t ri, rj;
+    uint32_t inter, uni;
+    int32_t cls;
+  };
+  constexpr size_t BS = 4096;
+  std::vector<Pre> pre(BS);
+  size_t blk0 = 0, blk1 = 0;
+  int64_t n_spec_used = 0;
+  auto find_ro = [&](int32_t x) {  // read-only root walk
+    while (nd[x].parent != x) x = nd[x].parent;
+    return x;
+  };
+  auto evaluate_block = [&](size_t from) {
+    flush_recent();  // the speculative pass reads `members` only
+    midflush = false;
+    blk0 = from;
+    blk1 = std::min(init_pos, from + BS);
+    std::memset(modbits, 0, sizeof(modbits));
+#pragma omp parallel for schedule(static, 64)
+    for (int64_t k = (int64_t)blk0; k < (int64_t)blk1; ++k) {
+      Pre& p = pre[(size_t)k - blk0];
+      const int32_t i = (int32_t)init[k].i, j = (int32_t)init[k].j;
+      if (nd[i].parent == i && nd[j].parent == j) {
+        p.cls = 0;
+        continue;
+      }
+      const int32_t ri = find_ro(i), rj = find_ro(j);
+      p.ri = ri;
+      p.rj = rj;
+      if (((nd[ri].sz | nd[rj].sz) & kDeleted) || ri == rj) {
+        p.cls = 1;
+        continue;
+      }
+      const uint32_t lo = (uint32_t)std::min(ri, rj), hi = (uint32_t)std::max(ri, rj);
+      if (is_candidate_big(((uint64_t)lo << 32) | hi)) {
+        p.cls = 2;
+        continue;
+      }
+      Cand c;
+      similarity(lo, hi, &c);
+      p.inter = c.inter;
+      p.uni = c.uni;
+      p.cls = 3;
+    }
+  };
+  constexpr size_t PF = 32, PF2 = 16, PF3 = 8;  // prefetch distances (sequential mode)
   while (nclusters > 0) {
     int32_t i, j;
     if (!zero_phase) {
       if (cur < init_pos && (extra.empty() || before(init[cur], extra.top()))) {
+        i = (int32_t)init[cur].i;
+        j = (int32_t)init[cur].j;
+        if (spec) {
+          if (cur >= blk1) evaluate_block(cur);
+          if (cur + PF < blk1 && pre[cur + PF - blk0].cls == 0) {  // merge-path pops read both nodes
+            __builtin_prefetch(&nd[init[cur + PF].i]);
+            __builtin_prefetch(&nd[init[cur + PF].j]);
+          }
+          const Pre& p = pre[cur - blk0];
+          ++cur;
+          if (p.cls == 1) {
+            ++n_spec_used;
+            continue;
+          }
+          if ((p.cls == 2 || p.cls == 3) && !is_mod(p.ri) && !is_mod(p.rj)) {
+            ++n_spec_used;
+            if (p.cls == 2) continue;
+            const uint32_t lo = (uint32_t)std::min(p.ri, p.rj), hi = (uint32_t)std::max(p.ri, p.rj);
+            const uint64_t key = ((uint64_t)lo << 32) | hi;
+            // re-inserted by an earlier pop of this block?
+            if (recent.contains(key) || (midflush && members.contains(key))) continue;
+            Cand c;
+            c.i = lo;
+            c.j = hi;
+            c.inter = p.inter;
+            c.uni = p.uni;
+            reinsert(c, key);
+            continue;
+          }
+          process(i, j);
+          continue;
+        }
         if (cur + PF < init_pos) {
           __builtin_prefetch(&nd[init[cur + PF].i]);
           __builtin_prefetch(&nd[init[cur + PF].j]);
@@ -344,8 +545,6 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
             }
           }
         }
-        i = (int32_t)init[cur].i;
-        j = (int32_t)init[cur].j;
         ++cur;
       } else if (!extra.empty()) {
         i = (int32_t)extra.top().i;
@@ -353,7 +552,9 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
         extra.pop();
       } else {
         zero_phase = true;
-        if (dbg) fprintf(stderr, "  J>0 phase %.3f s, %lld clusters left, %zu J=0 pairs\n", now() - t2, (long long)nclusters, zero_keys.size());
+        if (dbg)
+          fprintf(stderr, "  J>0 phase %.3f s, %lld clusters left, %zu J=0 pairs, %lld speculative results used\n",
+                  now() - t2, (long long)nclusters, zero_keys.size(), (long long)n_spec_used);
         for (size_t e = init_pos; e < (size_t)npairs; ++e) zero_keys.push_back(((uint64_t)init[e].i << 32) | init[e].j);
         __gnu_parallel::sort(zero_keys.begin(), zero_keys.end());
         continue;
@@ -364,53 +565,20 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
         i = (int32_t)extra.top().i;
         j = (int32_t)extra.top().j;
         extra.pop();
-        goto have_pair;
-      }
-      if (zc < zero_keys.size() && (zero_new.empty() || zero_keys[zc] < zero_new.top())) {
-        key = zero_keys[zc++];
-      } else if (!zero_new.empty()) {
-        key = zero_new.top();
-        zero_new.pop();
       } else {
-        break;  // every structure is empty
-      }
-      i = (int32_t)(key >> 32);
-      j = (int32_t)(key & 0xFFFFFFFFu);
-    }
-  have_pair:
-    if (nd[i].parent == i && nd[j].parent == j) {
-      if ((nd[i].sz | nd[j].sz) & kDeleted) continue;
-      // the larger cluster absorbs the smaller; equal sizes: smaller index (R6)
-      const bool i_wins = nd[i].sz > nd[j].sz || (nd[i].sz == nd[j].sz && i < j);
-      const int32_t w = i_wins ? i : j, l = i_wins ? j : i;
-      nd[l].parent = w;
-      nd[w].sz += nd[l].sz;  // R4
-      --nclusters;
-      if (nd[w].sz >= (uint32_t)threshold_size) {  // R7, R5
-        nd[w].sz |= kDeleted;
-        --nclusters;
-      }
-    } else {
-      i = root(i);
-      j = root(j);
-      if (((nd[i].sz | nd[j].sz) & kDeleted) || i == j) continue;
-      const uint32_t lo = (uint32_t)std::min(i, j), hi = (uint32_t)std::max(i, j);
-      const uint64_t key = ((uint64_t)lo << 32) | hi;
-      if (is_candidate(key)) continue;
-      Cand c;
-      similarity(lo, hi, &c);  // representing rows (R8)
-      members.insert(key);
-      ++n_reinsert;
-      if (c.inter > 0) {
-        extra.push(c);
-      } else {
-        ++n_zero;
-        if (zero_phase)
-          zero_new.push(key);
-        else
-          zero_keys.push_back(key);
+        if (zc < zero_keys.size() && (zero_new.empty() || zero_keys[zc] < zero_new.top())) {
+          key = zero_keys[zc++];
+        } else if (!zero_new.empty()) {
+          key = zero_new.top();
+          zero_new.pop();
+        } else {
+          break;  // every structure is empty
+        }
+        i = (int32_t)(key >> 32);
+        j = (int32_t)(key & 0xFFFFFFFFu);
       }
     }
+    process(i, j);
   }
   if (dbg)
     fprintf(stderr, "cluster_rows: set %.3f s, digests %.3f s, build %.3f s, sort %.3f s (sorted=%d), loop %.3f s, %lld re-inserted (%lld with J = 0)\n",

@@ -52,6 +52,17 @@ struct Frag<4> {
   __device__ __forceinline__ void store_cs(float* p) const { __stcs(reinterpret_cast<float4*>(p), v); }
 };
 template <>
+struct Frag<2> {
+  float2 v;
+  __device__ __forceinline__ void zero() { v = make_float2(0.f, 0.f); }
+  __device__ __forceinline__ void load_g(const float* p) { v = __ldg(reinterpret_cast<const float2*>(p)); }
+  __device__ __forceinline__ void load_cg(const float* p) { v = __ldcg(reinterpret_cast<const float2*>(p)); }
+  __device__ __forceinline__ void fma(float a, const Frag& b) { v.x = fmaf(a, b.v.x, v.x); v.y = fmaf(a, b.v.y, v.y); }
+  __device__ __forceinline__ void add(const Frag& b) { v.x += b.v.x; v.y += b.v.y; }
+  __device__ __forceinline__ void store(float* p) const { *reinterpret_cast<float2*>(p) = v; }
+  __device__ __forceinline__ void store_cs(float* p) const { __stcs(reinterpret_cast<float2*>(p), v); }
+};
+template <>
 struct Frag<1> {
   float v;
   __device__ __forceinline__ void zero() { v = 0.f; }
@@ -529,6 +540,178 @@ __global__ void __launch_bounds__(256, MINB) sddmm_task_kernel(
         }
       }
     }
+  }
+}
+
+// ------------------------------------------------------------------ phase D: register tiles
+// The ASpT dense tiles of panels of <= kRtMaxRows (8) rows (P:111 with a warp-sized panel).  One
+// warp owns one panel and keeps the accumulators of all its rows in registers (lane owns VEC
+// columns of each row): per dense column it gathers the B row ONCE (the column's header in the
+// entry stream) and adds it into every panel row that holds the column (row mask), so a column
+// shared by ρ rows costs one gather instead of ρ — the reuse ASpT gets from shared memory, here
+// without a staging copy or a shared-memory read per nnz (on B200 an LDS.128 of a staged row
+// costs the LSU data pipe as much as the L2 gather it replaces).  U columns are in flight.
+// Stream: api.cpp build_rt_stream (headers {col | kRtHeader, mask}, values {row, bits}, columns
+// never straddle a 32-entry batch).  Rows with dense nnz are written here; phase S (launched
+// after, same stream) read-modify-writes the rows that also have remainder nnz.  Each row's
+// dense nnz are added in slot order (count desc, column asc).
+template <int U, int VEC, int MINB>
+__global__ void __launch_bounds__(256, MINB) spmm_rtile_kernel(
+    const int4* __restrict__ units, int64_t n_units, const int2* __restrict__ ent,
+    const int32_t* __restrict__ dense_out, const float* __restrict__ B, uint32_t ldb, float* __restrict__ C,
+    int64_t ldc, int kw) {
+  constexpr int P = kRtMaxRows;
+  const int lane = threadIdx.x & 31;
+  const int64_t w = (int64_t)blockIdx.x * (blockDim.x >> 5) + __shfl_sync(FULL, threadIdx.x >> 5, 0);
+  if (w >= n_units) return;
+  int4 u = __ldg(units + w);  // {e0, e1, first position, rows}; warp-uniform via lane-0 shuffles
+  u.x = __shfl_sync(FULL, u.x, 0); u.y = __shfl_sync(FULL, u.y, 0);
+  u.z = __shfl_sync(FULL, u.z, 0); u.w = __shfl_sync(FULL, u.w, 0);
+  const bool kv = lane * VEC < kw;  // this lane's columns exist (last pass of a ragged K)
+  const char* Bk = reinterpret_cast<const char*>(B + (kv ? lane * VEC : 0));
+  Frag<VEC> acc[P];
+#pragma unroll
+  for (int r = 0; r < P; ++r) acc[r].zero();
+  for (int eb = u.x; eb < u.y; eb += 32) {
+    const int n = min(32, u.y - eb);
+    const int2 my = lane < n ? __ldcs(ent + eb + lane) : make_int2(0, 0);
+    unsigned hm = __ballot_sync(FULL, lane < n && my.x < 0);
+    while (hm) {
+      int hl[U];
+      Frag<VEC> b[U];
+#pragma unroll
+      for (int q = 0; q < U; ++q) {
+        hl[q] = hm ? __ffs(hm) - 1 : -1;
+        hm &= hm - 1;
+        if (hl[q] >= 0) {
+          const int c = __shfl_sync(FULL, my.x, hl[q]) & 0x7fffffff;
+          b[q].load_g(reinterpret_cast<const float*>(Bk + (uint64_t)(uint32_t)c * ldb));
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < U; ++q) {
+        if (hl[q] >= 0) {
+          const uint32_t mask = (uint32_t)__shfl_sync(FULL, my.y, hl[q]);
+          int pos = hl[q] + 1;
+#pragma unroll
+          for (int r = 0; r < P; ++r) {
+            if (mask & (1u << r)) {
+              acc[r].fma(__int_as_float(__shfl_sync(FULL, my.y, pos)), b[q]);
+              ++pos;
+            }
+          }
+        }
+      }
+    }
+  }
+  const int orow = lane < u.w ? __ldg(dense_out + u.z + lane) : -1;
+#pragma unroll
+  for (int r = 0; r < P; ++r) {
+    const int o = __shfl_sync(FULL, orow, r);
+    if (o >= 0 && kv) acc[r].store_cs(C + (int64_t)o * ldc + lane * VEC);
+  }
+}
+
+// SDDMM over the same register-tile stream: 8-lane groups (K = 32·NCH, lane holds NCH float4 of
+// an X row); group g keeps the X fragments of panel rows g and g+4 in registers, so per dense
+// column the Y row is gathered once (the four groups read the same addresses: one request) and
+// dotted with every panel row of the column's mask that the group owns; 3-step shuffle
+// reductions; out[oidx] = a·dot.
+template <int NCH, int MINB>
+__global__ void __launch_bounds__(256, MINB) sddmm_rtile_kernel(
+    const int4* __restrict__ units, int64_t n_units, const int2* __restrict__ ent, const int32_t* __restrict__ oidx,
+    const int32_t* __restrict__ pos_xrow, const float* __restrict__ X, int64_t ldx, const float* __restrict__ Y,
+    uint32_t ldy, int K, float* __restrict__ out, int accumulate) {
+  static_assert(kRtMaxRows == 8, "two panel rows per 8-lane group");
+  const int lane = threadIdx.x & 31, g = lane >> 3, lg = lane & 7;
+  const int64_t w = (int64_t)blockIdx.x * (blockDim.x >> 5) + __shfl_sync(FULL, threadIdx.x >> 5, 0);
+  if (w >= n_units) return;
+  int4 u = __ldg(units + w);
+  u.x = __shfl_sync(FULL, u.x, 0); u.y = __shfl_sync(FULL, u.y, 0);
+  u.z = __shfl_sync(FULL, u.z, 0); u.w = __shfl_sync(FULL, u.w, 0);
+  float4 x0[NCH], x1[NCH];
+  {
+    const int r0 = g, r1 = g + 4;
+    const float* p0 = X + (int64_t)(r0 < u.w ? __ldg(pos_xrow + u.z + r0) : 0) * ldx;
+    const float* p1 = X + (int64_t)(r1 < u.w ? __ldg(pos_xrow + u.z + r1) : 0) * ldx;
+#pragma unroll
+    for (int ch = 0; ch < NCH; ++ch) {
+      const int kk = ch * 32 + lg * 4;
+      x0[ch] = kk < K ? __ldg(reinterpret_cast<const float4*>(p0 + kk)) : make_float4(0.f, 0.f, 0.f, 0.f);
+      x1[ch] = kk < K ? __ldg(reinterpret_cast<const float4*>(p1 + kk)) : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+  }
+  const char* Yl = reinterpret_cast<const char*>(Y + lg * 4);
+  for (int eb = u.x; eb < u.y; eb += 32) {
+    const int n = min(32, u.y - eb);
+    const int2 my = lane < n ? __ldcs(ent + eb + lane) : make_int2(0, 0);
+    const int myo = lane < n ? __ldcs(oidx + eb + lane) : -1;
+    unsigned hm = __ballot_sync(FULL, lane < n && my.x < 0);
+    while (hm) {
+      const int h = __ffs(hm) - 1;
+      hm &= hm - 1;
+      const int c = __shfl_sync(FULL, my.x, h) & 0x7fffffff;
+      const uint32_t mask = (uint32_t)__shfl_sync(FULL, my.y, h);
+      float4 y[NCH];
+      const char* yp = Yl + (uint64_t)(uint32_t)c * ldy;
+#pragma unroll
+      for (int ch = 0; ch < NCH; ++ch)
+        y[ch] = (ch * 32 + lg * 4 < K) ? __ldg(reinterpret_cast<const float4*>(yp + ch * 128))
+                                       : make_float4(0.f, 0.f, 0.f, 0.f);
+      const bool has0 = (mask >> g) & 1u, has1 = (mask >> (g + 4)) & 1u;
+      float d0 = 0.f, d1 = 0.f;
+#pragma unroll
+      for (int ch = 0; ch < NCH; ++ch) {
+        d0 += fmaf(x0[ch].x, y[ch].x, fmaf(x0[ch].y, y[ch].y, fmaf(x0[ch].z, y[ch].z, x0[ch].w * y[ch].w)));
+        d1 += fmaf(x1[ch].x, y[ch].x, fmaf(x1[ch].y, y[ch].y, fmaf(x1[ch].z, y[ch].z, x1[ch].w * y[ch].w)));
+      }
+#pragma unroll
+      for (int off = 4; off > 0; off >>= 1) {
+        d0 += __shfl_xor_sync(FULL, d0, off);
+        d1 += __shfl_xor_sync(FULL, d1, off);
+      }
+      // entry lanes of rows g and g+4 in this column: after the header, rows ascending
+      const int p0 = h + 1 + __popc(mask & ((1u << g) - 1u));
+      const int p1 = h + 1 + __popc(mask & ((1u << (g + 4)) - 1u));
+      const float a0 = __int_as_float(__shfl_sync(FULL, my.y, p0 & 31));
+      const int o0 = __shfl_sync(FULL, myo, p0 & 31);
+      const float a1 = __int_as_float(__shfl_sync(FULL, my.y, p1 & 31));
+      const int o1 = __shfl_sync(FULL, myo, p1 & 31);
+      if (lg == 0) {  // K > 128: the host runs 128-column chunks, later ones add to out
+        if (has0) __stcs(out + o0, a0 * d0 + (accumulate ? __ldcg(out + o0) : 0.f));
+        if (has1) __stcs(out + o1, a1 * d1 + (accumulate ? __ldcg(out + o1) : 0.f));
+      }
+    }
+  }
+}
+
+// Scalar fallback of sddmm_rtile_kernel (unaligned operands or K % 4 != 0): one warp per panel
+// walks its stream; lanes split K; 5-step reduction.
+__global__ void __launch_bounds__(256) sddmm_rtile_scalar_kernel(
+    const int2* __restrict__ ent, const int32_t* __restrict__ oidx, const int4* __restrict__ units, int64_t n_units,
+    const int32_t* __restrict__ pos_xrow, const float* __restrict__ X, int64_t ldx, const float* __restrict__ Y,
+    int64_t ldy, int K, float* __restrict__ out) {
+  const int lane = threadIdx.x & 31;
+  const int64_t w = (int64_t)blockIdx.x * (blockDim.x >> 5) + __shfl_sync(FULL, threadIdx.x >> 5, 0);
+  if (w >= n_units) return;
+  const int4 u = units[w];
+  int col = 0, rem = 0;
+  for (int e = u.x; e < u.y; ++e) {
+    const int2 v = ent[e];
+    if (v.x < 0) {
+      col = v.x & 0x7fffffff;
+      rem = __popc((unsigned)v.y);
+      continue;
+    }
+    if (rem == 0) continue;  // padding
+    --rem;
+    const float* xr = X + (int64_t)pos_xrow[u.z + v.x] * ldx;
+    const float* yr = Y + (int64_t)col * ldy;
+    float d = 0.f;
+    for (int k = lane; k < K; k += 32) d = fmaf(xr[k], yr[k], d);
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) d += __shfl_xor_sync(FULL, d, off);
+    if (lane == 0) out[oidx[e]] = __int_as_float(v.y) * d;
   }
 }
 
@@ -1031,6 +1214,10 @@ int env_int(const char* name, int dflt) {
   const char* d = getenv(name);
   return d ? atoi(d) : dflt;
 }
+int rt_variant() {  // SR_RT_VARIANT (measurement knob): register-tile SpMM lane width / columns in flight
+  static const int v = env_int("SR_RT_VARIANT", 0);
+  return v;
+}
 bool task_kernels() {
   static const bool v = env_int("SR_PHASE_S", 1) != 0;
   return v;
@@ -1054,6 +1241,30 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
   constexpr int KC = LPG * VEC;
   constexpr int U = (LPG == 32) ? 8 : 4;  // gathers in flight per lane (phase S)
   constexpr int UD = 4;                   // shared-memory reads in flight per lane (phase D)
+  if (P.n_rt > 0) {  // register-tile phase D (panels of <= kRtMaxRows rows)
+    const unsigned grid = (unsigned)((P.n_rt + kSparseWarps - 1) / kSparseWarps);
+    if (P.profiling) SR_TRY(prof_begin(P, 5, s));
+    const int rv = rt_variant();
+    auto rk = [&](auto kern, int vec) {
+      const int pass = 32 * vec;
+      for (int64_t k0 = 0; k0 < K; k0 += pass)
+        kern<<<grid, kSparseWarps * 32, 0, s>>>(P.rt_units.p, P.n_rt, P.rt_ent.p, P.dense_out.p, B + k0,
+                                                 (uint32_t)(ldb * 4), C + k0, ldc, (int)std::min<int64_t>(pass, K - k0));
+    };
+    if constexpr (VEC == 4) {
+      switch (rv) {
+        case 1: rk(spmm_rtile_kernel<8, 4, 3>, 4); break;
+        case 2: rk(spmm_rtile_kernel<8, 2, 6>, 2); break;
+        case 3: rk(spmm_rtile_kernel<4, 2, 8>, 2); break;
+        default: rk(spmm_rtile_kernel<4, 4, 4>, 4); break;
+      }
+    } else {
+      rk(spmm_rtile_kernel<8, 1, 8>, 1);
+    }
+    SR_CUDA_TRY(cudaGetLastError());
+    if (P.profiling) SR_TRY(prof_end(P, s));
+    ++*launches;
+  }
   if (P.n_units > 0) {
     const int TW = P.tile_cols;
     const size_t smem =
@@ -1131,6 +1342,22 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
   constexpr int KC = LPG * VEC;
   constexpr int U = (LPG == 32) ? 4 : 2;
   constexpr int NCH_D = (LPG == 32) ? 1 : NCH;  // dense: whole K per pass unless K > 256
+  if (P.n_rt > 0) {  // register-tile phase D: 128-column chunks (vector path) or a scalar fallback
+    if (P.profiling) SR_TRY(prof_begin(P, 6, s));
+    const unsigned grid = (unsigned)((P.n_rt + kSparseWarps - 1) / kSparseWarps);
+    if constexpr (VEC == 4) {
+      for (int64_t k0 = 0; k0 < K; k0 += 128)
+        sddmm_rtile_kernel<4, 4><<<grid, kSparseWarps * 32, 0, s>>>(
+            P.rt_units.p, P.n_rt, P.rt_ent.p, P.rt_oidx.p, P.pos_xrow.p, X + k0, ldx, Y + k0, (uint32_t)(ldy * 4),
+            (int)std::min<int64_t>(128, K - k0), out, k0 > 0 ? 1 : 0);
+    } else {
+      sddmm_rtile_scalar_kernel<<<grid, kSparseWarps * 32, 0, s>>>(P.rt_ent.p, P.rt_oidx.p, P.rt_units.p, P.n_rt,
+                                                                    P.pos_xrow.p, X, ldx, Y, ldy, (int)K, out);
+    }
+    SR_CUDA_TRY(cudaGetLastError());
+    if (P.profiling) SR_TRY(prof_end(P, s));
+    ++*launches;
+  }
   if (P.n_units > 0) {
     const int TW = P.tile_cols;
     const size_t smem =

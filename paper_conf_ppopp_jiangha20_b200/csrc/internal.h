@@ -134,6 +134,9 @@ struct __align__(16) DUnit {
   int32_t split;      // -1: the unit covers its whole panel; else its partial-sum slot
   int32_t pad0, pad1, pad2;
 };
+constexpr int kRtMaxRows = 8;                        // register-tile engine: panel rows
+constexpr int64_t kRtMaxPanelEntries = 4096;         // larger panels stay on the TMA engine
+constexpr int32_t kRtHeader = (int32_t)0x80000000u;  // marks a column header entry
 constexpr int kMaxUnitTiles = 8;
 constexpr int kMaxExecTile = 64;
 constexpr int kMaxTileEntries = 384;  // SpMM: 3 stages + blob ring must fit twice per SM
@@ -172,6 +175,11 @@ struct DevPlan {
   int64_t n_dslots = 0;
   DevBuf<float> dscratch;     // n_dslots × panel_rows × dscratch_k
   int64_t dscratch_k = 0;
+  // phase D, register-tile engine (panels of <= kRtMaxRows rows; api.cpp: build_rt_stream)
+  int64_t n_rt = 0;
+  DevBuf<int4> rt_units;      // one warp per panel: {e0, e1, first position, rows}
+  DevBuf<int2> rt_ent;        // column headers {col | kRtHeader, row mask} + {row, value bits}
+  DevBuf<int32_t> rt_oidx;    // SDDMM output index per value entry (-1: header / padding)
   DevBuf<int32_t> pos_xrow;   // position -> original row
   DevBuf<int32_t> pos_out;    // position -> SpMM output row
   DevBuf<int32_t> dense_out;  // position -> SpMM output row if the row has dense nnz, else -1

@@ -4,10 +4,9 @@
 //   minhash_bandkeys : warp per non-empty row; lane owns hash functions s = lane + 32t,
 //                      sweeps the row's columns (broadcast by shuffle) keeping running minima,
 //                      then writes one u64 band key per band (bsize 1 or 2: the exact tuple).
-//   all bands at once: one stable radix sort of (band key, band|row) — equal keys of different
-//                      bands stay grouped by band, members ascending; run heads on (key, band)
-//                      -> bucket starts and sizes; chunk cap (R14) -> pair counts; emit_pairs_all:
-//                      thread per bucket member, O(1) output offset.  Two host syncs in total.
+//   per band         : radix sort (key, row) — stable, so bucket members stay ascending;
+//                      run-length encode -> bucket sizes; chunk cap (R14) -> pair counts;
+//                      emit_pairs: thread per bucket member, O(1) output offset.
 //   all bands        : radix sort packed pairs + unique  -> E (union over bands, R13/R14).
 //   pair_jaccard     : thread per pair, sorted-list merge (binary-search when lopsided).
 //   heap order       : sort by (J desc, pair asc) through an exact 64-bit fixed-point key
@@ -16,6 +15,9 @@
 #include <cub/cub.cuh>
 
 #include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <vector>
 
 #include "internal.h"
@@ -94,42 +96,19 @@ __device__ __forceinline__ int64_t chunk_pairs(int64_t s, int64_t C) {
   return f * (C * (C - 1) / 2) + r * (r - 1) / 2;
 }
 
-
-
-
-
-// All bands in one pass: after one stable radix sort of every (band key, band·L + t) pair by
-// the 64-bit key, equal keys of different bands stay grouped by band (the input is band-major and
-// the sort stable) and rows ascend inside each group, so a bucket is a maximal run of equal
-// (key, band) with its members ascending — exactly O5's bucket.
-__global__ void run_heads(const uint64_t* __restrict__ k, const uint32_t* __restrict__ v, int64_t n, int shift,
-                          uint8_t* __restrict__ head) {
+__global__ void run_pair_counts(const int32_t* __restrict__ run_len, int64_t nruns, int64_t C,
+                                int64_t* __restrict__ npairs) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= n) return;
-  head[i] = (i == 0 || k[i] != k[i - 1] || (v[i] >> shift) != (v[i - 1] >> shift)) ? 1 : 0;
+  if (i < nruns) npairs[i] = chunk_pairs(run_len[i], C);
 }
 
-__global__ void run_lengths(const int64_t* __restrict__ start, int64_t nruns, int64_t n, int32_t* __restrict__ len,
-                            int64_t* __restrict__ npairs, int64_t C) {
-  const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (r > nruns) return;
-  if (r == nruns) {
-    npairs[r] = 0;
-    return;
-  }
-  const int64_t l = (r + 1 < nruns ? start[r + 1] : n) - start[r];
-  len[r] = (int32_t)l;
-  npairs[r] = chunk_pairs(l, C);
-}
-
-// element x of run r emits the pairs (x, y), y after x in its chunk (as emit_pairs); members are
-// live ids t (value & mask), ascending within the run
-__global__ void emit_pairs_all(const int32_t* __restrict__ run_of, const int64_t* __restrict__ run_start,
-                               const int32_t* __restrict__ run_len, const int64_t* __restrict__ run_off,
-                               const uint32_t* __restrict__ vals_sorted, uint32_t mask,
-                               const int32_t* __restrict__ live, int64_t n, int64_t C, uint64_t* __restrict__ out) {
+// element x of run r (start s0, size sz) emits pairs (x, y) for y after x in its chunk
+__global__ void emit_pairs(const int32_t* __restrict__ run_of, const int64_t* __restrict__ run_start,
+                           const int32_t* __restrict__ run_len, const int64_t* __restrict__ run_off,
+                           const int32_t* __restrict__ vals_sorted, const int32_t* __restrict__ live,
+                           int64_t L, int64_t C, uint64_t* __restrict__ out) {
   const int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (x >= n) return;
+  if (x >= L) return;
   const int32_t r = run_of[x];
   const int64_t sz = run_len[r];
   if (sz < 2) return;
@@ -141,35 +120,51 @@ __global__ void emit_pairs_all(const int32_t* __restrict__ run_of, const int64_t
   const int64_t clen = min(cap, sz - cs);
   const int64_t k = lx - cs;
   int64_t o = run_off[r] + chunk * (cap * (cap - 1) / 2) + k * (clen - 1) - k * (k - 1) / 2;
-  const uint64_t me = (uint64_t)(uint32_t)live[vals_sorted[x] & mask];
+  const uint64_t me = (uint64_t)(uint32_t)live[vals_sorted[x]];
   for (int64_t y = x + 1; y < s0 + cs + clen; ++y) {
-    const uint64_t other = (uint64_t)(uint32_t)live[vals_sorted[y] & mask];
-    out[o++] = (me << 32) | other;
+    const uint64_t other = (uint64_t)(uint32_t)live[vals_sorted[y]];
+    out[o++] = (me << 32) | other;  // live ids ascending within a bucket => me < other
   }
 }
 
-__global__ void band_iota(uint32_t* __restrict__ v, int64_t L, int shift, int64_t n) {
-  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i < n) v[i] = ((uint32_t)(i / L) << shift) | (uint32_t)(i % L);
-}
-
-__global__ void mark_runs64(const int64_t* __restrict__ run_start, const int32_t* __restrict__ run_len,
-                            int64_t nruns, int32_t* __restrict__ run_of) {
+__global__ void mark_runs(const int64_t* __restrict__ run_start, const int32_t* __restrict__ run_len,
+                          int64_t nruns, int32_t* __restrict__ run_of) {
   const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (r >= nruns) return;
   const int64_t s0 = run_start[r];
   for (int32_t t = 0; t < run_len[r]; ++t) run_of[s0 + t] = (int32_t)r;
 }
 
-__global__ void iota_i64(int64_t* a, int64_t n) {
+__global__ void to_int64(const int32_t* __restrict__ a, int64_t n, int64_t* __restrict__ b) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i < n) a[i] = i;
+  if (i < n) b[i] = a[i];
 }
 
+// exact order-preserving key of J = n/u: floor(2^64·n/u) (n < u), all-ones for J = 1; stored
+// complemented so an ascending sort gives J descending
+__device__ __forceinline__ uint64_t jaccard_key(uint32_t n, uint32_t u) {
+  uint64_t key;
+  if (u == 0 || n == 0) {
+    key = 0;
+  } else if (n >= u) {
+    key = ~0ull;
+  } else {
+    const uint64_t hi = ((uint64_t)n << 32) / u, r1 = ((uint64_t)n << 32) % u;
+    const uint64_t lo = (r1 << 32) / u;
+    key = (hi << 32) | lo;
+  }
+  return ~key;
+}
+
+constexpr int64_t kLongPair = 2048;  // pairs with more column entries go to the warp kernel
+
+// thread per pair: sorted-list merge (binary search when lopsided); pairs whose two lists hold
+// more than kLongPair entries are queued for pair_jaccard_long (one warp each), so a few hub-row
+// pairs (R-MAT rows reach 39,705 nnz) no longer serialise whole warps
 __global__ void pair_jaccard(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
                              const uint64_t* __restrict__ pairs, int64_t E,
                              uint32_t* __restrict__ inter, uint32_t* __restrict__ uni,
-                             uint64_t* __restrict__ jkey) {
+                             uint64_t* __restrict__ jkey, int64_t* __restrict__ long_idx, int* __restrict__ n_long) {
   const int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (e >= E) return;
   const uint64_t pr = pairs[e];
@@ -177,6 +172,10 @@ __global__ void pair_jaccard(const int64_t* __restrict__ rowptr, const int32_t* 
   const int32_t *a = col + rowptr[i], *ae = col + rowptr[i + 1];
   const int32_t *b = col + rowptr[j], *be = col + rowptr[j + 1];
   int64_t na = ae - a, nb = be - b;
+  if (na + nb > kLongPair) {
+    long_idx[atomicAdd(n_long, 1)] = e;
+    return;
+  }
   if (na > nb) {
     const int32_t* t = a; a = b; b = t;
     t = ae; ae = be; be = t;
@@ -206,18 +205,46 @@ __global__ void pair_jaccard(const int64_t* __restrict__ rowptr, const int32_t* 
   const uint32_t u = (uint32_t)(na + nb - n);
   inter[e] = n;
   uni[e] = u;
-  // exact order-preserving key of J = n/u: floor(2^64·n/u) (n < u), all-ones for J = 1
-  uint64_t key;
-  if (u == 0 || n == 0) {
-    key = 0;
-  } else if (n >= u) {
-    key = ~0ull;
-  } else {
-    const uint64_t hi = ((uint64_t)n << 32) / u, r1 = ((uint64_t)n << 32) % u;
-    const uint64_t lo = (r1 << 32) / u;
-    key = (hi << 32) | lo;
+  jkey[e] = jaccard_key(n, u);
+}
+
+// one warp per queued long pair: lanes stride over the shorter list and binary-search the longer
+__global__ void pair_jaccard_long(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
+                                  const uint64_t* __restrict__ pairs, const int64_t* __restrict__ long_idx,
+                                  const int* __restrict__ n_long, uint32_t* __restrict__ inter,
+                                  uint32_t* __restrict__ uni, uint64_t* __restrict__ jkey) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
+  const int nl = *n_long;
+  for (int64_t w = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); w < nl; w += nw) {
+    const int64_t e = long_idx[w];
+    const uint64_t pr = pairs[e];
+    const int64_t i = (int64_t)(pr >> 32), j = (int64_t)(pr & 0xFFFFFFFFu);
+    const int32_t *a = col + rowptr[i], *b = col + rowptr[j];
+    int64_t na = rowptr[i + 1] - rowptr[i], nb = rowptr[j + 1] - rowptr[j];
+    if (na > nb) {
+      const int32_t* t = a; a = b; b = t;
+      const int64_t tn = na; na = nb; nb = tn;
+    }
+    uint32_t n = 0;
+    for (int64_t t = lane; t < na; t += 32) {
+      const int32_t v = a[t];
+      int64_t lo = 0, cnt = nb;
+      while (cnt > 0) {
+        const int64_t h = cnt >> 1;
+        if (b[lo + h] < v) { lo += h + 1; cnt -= h + 1; } else { cnt = h; }
+      }
+      n += (lo < nb && b[lo] == v);
+    }
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) n += __shfl_xor_sync(0xffffffffu, n, off);
+    if (lane == 0) {
+      const uint32_t u = (uint32_t)(na + nb - n);
+      inter[e] = n;
+      uni[e] = u;
+      jkey[e] = jaccard_key(n, u);
+    }
   }
-  jkey[e] = ~key;  // ascending sort of ~key == J descending
 }
 
 __global__ void iota_u32(uint32_t* a, int64_t n) {
@@ -244,6 +271,16 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
                    const sr_reorder_params& p, cudaStream_t s, std::vector<uint64_t>& pairs_by_j,
                    std::vector<uint32_t>& inter_h, std::vector<uint32_t>& uni_h, int64_t* E_out,
                    std::vector<uint64_t>* pairs_by_key) {
+  const bool dbg = getenv("SR_DEBUG_LSH") != nullptr;  // per-phase wall times (syncs the stream)
+  double tl = 0;
+  auto lap = [&](const char* what) {
+    if (!dbg) return;
+    cudaStreamSynchronize(s);
+    const double t = std::chrono::duration<double>(std::chrono::steady_clock::now().time_since_epoch()).count();
+    if (tl > 0) fprintf(stderr, "lsh: %-28s %.4f s\n", what, t - tl);
+    tl = t;
+  };
+  lap("start");
   pairs_by_j.clear();
   inter_h.clear();
   uni_h.clear();
@@ -269,6 +306,7 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
   SR_TRY(d_live.upload(live, s));
   SR_TRY(d_a.upload(ha, s));
   SR_TRY(d_b.upload(hb, s));
+  lap("host prep + uploads");
   DevBuf<uint64_t> keys;
   SR_TRY(keys.alloc((size_t)nb * L));
   {
@@ -285,27 +323,28 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
 #undef SR_MH
     SR_CUDA_TRY(cudaGetLastError());
   }
-  // all bands at once: one stable radix sort of (key, band·2^shift | t), run heads on
-  // (key, band), run starts by a flagged select, chunk-capped pair counts (R14), one scan, one
-  // emit launch; two host syncs in total (run count, pair count)
-  const int64_t NB = (int64_t)nb * L;
-  int shift = 1, band_bits = 0;
-  while ((int64_t(1) << shift) < L) ++shift;
-  while ((1 << band_bits) < nb) ++band_bits;
-  if (shift + band_bits > 32) {
-    set_error("lsh_candidates: non-empty rows x bands exceed the 32-bit (band, row) index of the one-pass banding");
-    return SR_EUNSUPPORTED;
-  }
+  lap("minhash");
+  // per band: sort, bucket, emit
   DevBuf<uint64_t> kout;
-  DevBuf<uint32_t> vin, vout;
-  DevBuf<uint8_t> head;
-  DevBuf<int64_t> idx, run_start, run_npairs, run_off, nruns_d;
-  DevBuf<int32_t> run_len, run_of;
-  SR_TRY(kout.alloc(NB));
-  SR_TRY(vin.alloc(NB));
-  SR_TRY(vout.alloc(NB));
-  band_iota<<<blocks(NB, 256), 256, 0, s>>>(vin.p, L, shift, NB);
-  SR_CUDA_TRY(cudaGetLastError());
+  DevBuf<int32_t> vin, vout, run_len, run_of, nruns_d;
+  DevBuf<uint64_t> run_key;
+  DevBuf<int64_t> run_start, run_npairs, run_off;
+  SR_TRY(kout.alloc(L));
+  SR_TRY(vin.alloc(L));
+  SR_TRY(vout.alloc(L));
+  SR_TRY(run_len.alloc(L));
+  SR_TRY(run_of.alloc(L));
+  SR_TRY(run_key.alloc(L));
+  SR_TRY(run_start.alloc(L + 1));
+  SR_TRY(run_npairs.alloc(L + 1));
+  SR_TRY(run_off.alloc(L + 1));
+  SR_TRY(nruns_d.alloc(1));
+  {
+    std::vector<int32_t> iota((size_t)L);
+    for (int64_t t = 0; t < L; ++t) iota[t] = (int32_t)t;
+    SR_CUDA_TRY(cudaMemcpyAsync(vin.p, iota.data(), L * sizeof(int32_t), cudaMemcpyHostToDevice, s));
+    SR_CUDA_TRY(cudaStreamSynchronize(s));
+  }
   DevBuf<uint8_t> temp;
   size_t temp_bytes = 0;
   auto ensure_temp = [&](size_t need) -> int {
@@ -315,66 +354,66 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
     }
     return SR_OK;
   };
-  {
-    size_t need = 0;
-    cub::DeviceRadixSort::SortPairs(nullptr, need, keys.p, kout.p, vin.p, vout.p, NB, 0, 64, s);
-    SR_TRY(ensure_temp(need));
-    need = temp_bytes;
-    SR_CUDA_TRY(cub::DeviceRadixSort::SortPairs(temp.p, need, keys.p, kout.p, vin.p, vout.p, NB, 0, 64, s));
-  }
-  keys.release();
-  vin.release();
-  SR_TRY(head.alloc(NB));
-  run_heads<<<blocks(NB, 256), 256, 0, s>>>(kout.p, vout.p, NB, shift, head.p);
-  SR_CUDA_TRY(cudaGetLastError());
-  SR_TRY(idx.alloc(NB));
-  SR_TRY(run_start.alloc(NB));
-  SR_TRY(nruns_d.alloc(1));
-  iota_i64<<<blocks(NB, 256), 256, 0, s>>>(idx.p, NB);
-  {
-    size_t need = 0;
-    cub::DeviceSelect::Flagged(nullptr, need, idx.p, head.p, run_start.p, nruns_d.p, NB, s);
-    SR_TRY(ensure_temp(need));
-    need = temp_bytes;
-    SR_CUDA_TRY(cub::DeviceSelect::Flagged(temp.p, need, idx.p, head.p, run_start.p, nruns_d.p, NB, s));
-  }
-  int64_t nruns = 0;
-  SR_CUDA_TRY(cudaMemcpyAsync(&nruns, nruns_d.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
-  SR_CUDA_TRY(cudaStreamSynchronize(s));
-  kout.release();
-  head.release();
-  idx.release();
-  const int64_t C = p.max_bucket;
   DevBuf<uint64_t> allpairs;
-  int64_t n_pairs = 0;
-  if (nruns < NB) {  // some bucket has two or more rows
-    SR_TRY(run_len.alloc(nruns));
-    SR_TRY(run_npairs.alloc(nruns + 1));
-    SR_TRY(run_off.alloc(nruns + 1));
-    SR_TRY(run_of.alloc(NB));
-    run_lengths<<<blocks(nruns + 1, 256), 256, 0, s>>>(run_start.p, nruns, NB, run_len.p, run_npairs.p, C);
-    mark_runs64<<<blocks(nruns, 256), 256, 0, s>>>(run_start.p, run_len.p, nruns, run_of.p);
-    SR_CUDA_TRY(cudaGetLastError());
+  int64_t cap_pairs = 0, n_pairs = 0;
+  const int64_t C = p.max_bucket;
+  for (int band = 0; band < nb; ++band) {
     size_t need = 0;
-    cub::DeviceScan::ExclusiveSum(nullptr, need, run_npairs.p, run_off.p, nruns + 1, s);
+    cub::DeviceRadixSort::SortPairs(nullptr, need, keys.p + (int64_t)band * L, kout.p, vin.p, vout.p, (int)L, 0, 64, s);
     SR_TRY(ensure_temp(need));
     need = temp_bytes;
-    SR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(temp.p, need, run_npairs.p, run_off.p, nruns + 1, s));
-    SR_CUDA_TRY(cudaMemcpyAsync(&n_pairs, run_off.p + nruns, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    SR_CUDA_TRY(cub::DeviceRadixSort::SortPairs(temp.p, need, keys.p + (int64_t)band * L, kout.p, vin.p,
+                                                vout.p, (int)L, 0, 64, s));
+    need = 0;
+    cub::DeviceRunLengthEncode::Encode(nullptr, need, kout.p, run_key.p, run_len.p, nruns_d.p, (int)L, s);
+    SR_TRY(ensure_temp(need));
+    need = temp_bytes;
+    SR_CUDA_TRY(cub::DeviceRunLengthEncode::Encode(temp.p, need, kout.p, run_key.p, run_len.p, nruns_d.p,
+                                                   (int)L, s));
+    int32_t nruns = 0;
+    SR_CUDA_TRY(cudaMemcpyAsync(&nruns, nruns_d.p, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
     SR_CUDA_TRY(cudaStreamSynchronize(s));
-    if (n_pairs > 0) {
-      SR_TRY(allpairs.alloc(n_pairs));
-      emit_pairs_all<<<blocks(NB, 256), 256, 0, s>>>(run_of.p, run_start.p, run_len.p, run_off.p, vout.p,
-                                                    (uint32_t)((1u << shift) - 1), d_live.p, NB, C, allpairs.p);
-      SR_CUDA_TRY(cudaGetLastError());
+    if (nruns == L) continue;  // every bucket is a singleton
+    // run starts = exclusive sum of lengths (int64)
+    to_int64<<<blocks(nruns, 256), 256, 0, s>>>(run_len.p, nruns, run_npairs.p);
+    need = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, need, run_npairs.p, run_start.p, (int)nruns + 0, s);
+    SR_TRY(ensure_temp(need));
+    need = temp_bytes;
+    SR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(temp.p, need, run_npairs.p, run_start.p, (int)nruns, s));
+    mark_runs<<<blocks(nruns, 256), 256, 0, s>>>(run_start.p, run_len.p, nruns, run_of.p);
+    run_pair_counts<<<blocks(nruns, 256), 256, 0, s>>>(run_len.p, nruns, C, run_npairs.p);
+    SR_CUDA_TRY(cudaMemsetAsync(run_npairs.p + nruns, 0, sizeof(int64_t), s));
+    need = 0;
+    cub::DeviceScan::ExclusiveSum(nullptr, need, run_npairs.p, run_off.p, (int)nruns + 1, s);
+    SR_TRY(ensure_temp(need));
+    need = temp_bytes;
+    SR_CUDA_TRY(cub::DeviceScan::ExclusiveSum(temp.p, need, run_npairs.p, run_off.p, (int)nruns + 1, s));
+    int64_t band_pairs = 0;
+    SR_CUDA_TRY(cudaMemcpyAsync(&band_pairs, run_off.p + nruns, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    SR_CUDA_TRY(cudaStreamSynchronize(s));
+    if (band_pairs == 0) continue;
+    if (n_pairs + band_pairs > cap_pairs) {
+      int64_t ncap = std::max<int64_t>(2 * cap_pairs, n_pairs + band_pairs);
+      ncap = std::max<int64_t>(ncap, 1 << 20);
+      DevBuf<uint64_t> bigger;
+      SR_TRY(bigger.alloc(ncap));
+      if (n_pairs)
+        SR_CUDA_TRY(cudaMemcpyAsync(bigger.p, allpairs.p, n_pairs * sizeof(uint64_t),
+                                    cudaMemcpyDeviceToDevice, s));
+      SR_CUDA_TRY(cudaStreamSynchronize(s));
+      std::swap(bigger.p, allpairs.p);
+      std::swap(bigger.n, allpairs.n);
+      cap_pairs = ncap;
     }
+    // run_off is relative to this band: shift output pointer
+    emit_pairs<<<blocks(L, 256), 256, 0, s>>>(run_of.p, run_start.p, run_len.p, run_off.p, vout.p, d_live.p,
+                                              L, C, allpairs.p + n_pairs);
+    SR_CUDA_TRY(cudaGetLastError());
+    n_pairs += band_pairs;
   }
-  run_of.release();
-  run_len.release();
-  run_npairs.release();
-  run_off.release();
-  run_start.release();
-  vout.release();
+  lap("bands");
+  keys.release();
   if (n_pairs == 0) return SR_OK;
   // union over bands: sort + unique
   DevBuf<uint64_t> sorted, uniq;
@@ -395,11 +434,12 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
     need = temp_bytes;
     SR_CUDA_TRY(cub::DeviceSelect::Unique(temp.p, need, sorted.p, allpairs.p, nuniq.p, n_pairs, s));
   }
+  lap("pair sort + unique");
   int64_t E = 0;
   SR_CUDA_TRY(cudaMemcpyAsync(&E, nuniq.p, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
   SR_CUDA_TRY(cudaStreamSynchronize(s));
   sorted.release();
-  if (pairs_by_key) {  // the unique pairs in key order: the clustering's membership index (R9)
+  if (pairs_by_key && E > (int64_t(1) << 26)) {  // the clustering's membership index above 2^26 pairs (R9)
     pairs_by_key->resize((size_t)E);
     SR_CUDA_TRY(cudaMemcpyAsync(pairs_by_key->data(), allpairs.p, E * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
   }
@@ -412,7 +452,15 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
   SR_TRY(jkey_out.alloc(E));
   SR_TRY(idx_in.alloc(E));
   SR_TRY(idx_out.alloc(E));
-  pair_jaccard<<<blocks(E, 256), 256, 0, s>>>(d_rowptr.p, d_col.p, allpairs.p, E, d_inter.p, d_uni.p, jkey.p);
+  DevBuf<int64_t> long_idx;
+  DevBuf<int> n_long;
+  SR_TRY(long_idx.alloc(E));
+  SR_TRY(n_long.alloc(1));
+  SR_CUDA_TRY(cudaMemsetAsync(n_long.p, 0, sizeof(int), s));
+  pair_jaccard<<<blocks(E, 256), 256, 0, s>>>(d_rowptr.p, d_col.p, allpairs.p, E, d_inter.p, d_uni.p, jkey.p,
+                                              long_idx.p, n_long.p);
+  pair_jaccard_long<<<1184, 256, 0, s>>>(d_rowptr.p, d_col.p, allpairs.p, long_idx.p, n_long.p, d_inter.p, d_uni.p,
+                                         jkey.p);
   iota_u32<<<blocks(E, 256), 256, 0, s>>>(idx_in.p, E);
   SR_CUDA_TRY(cudaGetLastError());
   {
@@ -428,6 +476,7 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
   SR_TRY(u2.alloc(E));
   gather_by<<<blocks(E, 256), 256, 0, s>>>(idx_out.p, E, allpairs.p, d_inter.p, d_uni.p, p2.p, i2.p, u2.p);
   SR_CUDA_TRY(cudaGetLastError());
+  lap("jaccard + heap sort");
   pairs_by_j.resize((size_t)E);
   inter_h.resize((size_t)E);
   uni_h.resize((size_t)E);
@@ -435,6 +484,7 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
   SR_CUDA_TRY(cudaMemcpyAsync(inter_h.data(), i2.p, E * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
   SR_CUDA_TRY(cudaMemcpyAsync(uni_h.data(), u2.p, E * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
   SR_CUDA_TRY(cudaStreamSynchronize(s));
+  lap("D2H");
   *E_out = E;
   return SR_OK;
 }

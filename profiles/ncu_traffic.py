@@ -3,7 +3,10 @@ kernels from an `ncu --set full ... --page raw --csv` export and merge it into
 profiles/ncu_traffic.json, keyed "<config>_K<K>_<kernel kind>" (bench.py reads it into the
 roofline `traffic` field).
 
-  python profiles/ncu_traffic.py <raw.csv> <config> <K> [source-tag]
+  python profiles/ncu_traffic.py <raw.csv> <config> <K> [source-tag] [kernel-sig]
+
+kernel-sig is bench.kernel_source_sig() of the sources the capture ran (write it on the GPU box
+next to the capture); bench.py uses a record only when it matches the current sources.
 """
 import csv
 import json
@@ -12,11 +15,12 @@ import sys
 
 KINDS = {"spmm_dense_kernel": "spmm_dense_tiles", "spmm_sparse_kernel": "spmm_sparse_rows",
          "spmm_task_kernel": "spmm_sparse_rows", "sddmm_dense_kernel": "sddmm_dense_tiles",
-         "sddmm_sparse_kernel": "sddmm_sparse_rows", "sddmm_task_kernel": "sddmm_sparse_rows"}
+         "sddmm_sparse_kernel": "sddmm_sparse_rows", "sddmm_task_kernel": "sddmm_sparse_rows",
+         "spmm_rtile_kernel": "spmm_register_tiles", "sddmm_rtile_kernel": "sddmm_register_tiles"}
 UNIT = {"byte": 1.0, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
 
 
-def main(path, config, K, tag=""):
+def main(path, config, K, tag="", sig=None):
     rows = list(csv.reader(open(path)))
     hdr, units, data = rows[0], rows[1], rows[2:]
     ix = {h: i for i, h in enumerate(hdr)}
@@ -33,6 +37,8 @@ def main(path, config, K, tag=""):
         t = float(d[ix["gpu__time_duration.sum"]]) * {"nsecond": 1e-9, "ns": 1e-9, "usecond": 1e-6, "us": 1e-6,
                                                        "msecond": 1e-3, "ms": 1e-3}[units[ix["gpu__time_duration.sum"]]]
         rec = {"bytes": total, "ncu_duration_s": t, "source": tag or os.path.basename(path)}
+        if sig:
+            rec["kernel_sig"] = sig
         for m, key in (("lts__t_sector_hit_rate.pct", "l2_hit_pct"), ("l1tex__t_sector_hit_rate.pct", "l1_hit_pct")):
             if m in ix and d[ix[m]] not in ("", "n/a"):
                 rec[key] = float(d[ix[m]])

@@ -56,6 +56,7 @@ def main():
     force = dict(siglen=32, bsize=2, seed=4, max_bucket=0, threshold_size=256, panel_rows=16, dense_min=2,
                  mode=sr.FORCE, tile_cols=16)
     run(tiny, sr.default_params(**force), (32, 128))
+    run(tiny, sr.default_params(**dict(force, panel_rows=8)), (32, 36, 128, 132))  # register-tile phase D
     H = matrix_with_long_rows_and_hub()
     M = run(H, sr.default_params(**force), (32, 128, 256))
     st = M.stats()

@@ -127,11 +127,13 @@ def test_auto_decision_threshold_plan(env, oracle, case):
 
 
 # ------------------------------------------------------------------ numerics over the plan
+@pytest.mark.parametrize("panel", [8, 16])
 @pytest.mark.parametrize("K", [1, 3, 4, 8, 32, 36, 64, 128, 132, 256])
-def test_k_sweep_forced_plan(env, oracle, K):
+def test_k_sweep_forced_plan(env, oracle, K, panel):
+    """panel 16: phase D on the TMA shared-memory engine; panel 8: the register-tile engine."""
     sr, _ = env
     A = g.random_csr(700, 500, 0.03, 5, empty_frac=0.1)
-    M, B, X, Y, C, out = _run(env, A, K, sr.default_params(**_plan_kw(16, 1, 8), tile_cols=8))
+    M, B, X, Y, C, out = _run(env, A, K, sr.default_params(**_plan_kw(panel, 1, 8), tile_cols=8))
     assert M.stats()["dense1"] > 0
     _spmm_check(oracle, A, B, C)
     _sddmm_check(oracle, A, X, Y, out)
@@ -166,7 +168,8 @@ def test_long_rows_split_and_rmw(env, oracle):
         cols.append(hub)
     rowptr, colidx = g._from_coo(n, m, np.concatenate(rows), np.concatenate(cols))
     A = g.CSR(n, m, rowptr, colidx, g._uniform_vals(colidx.size, 3))
-    for params in (None, sr.default_params(**_plan_kw(16, 1, 8)), sr.default_params(**_plan_kw(16, 2, 0))):
+    for params in (None, sr.default_params(**_plan_kw(16, 1, 8)), sr.default_params(**_plan_kw(16, 2, 0)),
+                   sr.default_params(**_plan_kw(8, 1, 8))):
         for K in (32, 128, 256):  # 256: two 128-column passes of the SpMM task kernel
             M, B, X, Y, C, out = _run(env, A, K, params)
             _spmm_check(oracle, A, B, C)
@@ -281,8 +284,9 @@ def test_bad_params(env):
 
 
 # ------------------------------------------------------------------ sharded plans on one GPU
+@pytest.mark.parametrize("panel", [8, 16])
 @pytest.mark.parametrize("world", [2, 3])
-def test_shard_simulation(env, oracle, world):
+def test_shard_simulation(env, oracle, world, panel):
     """Run every shard's plan on the same GPU and reassemble (SURVEY §4 tier 4a)."""
     sr, torch = env
     A = g.random_csr(500, 300, 0.03, 21, empty_frac=0.1)
@@ -295,7 +299,7 @@ def test_shard_simulation(env, oracle, world):
     ref_cuts = None
     for r in range(world):
         M = sr.SparseMatrix.from_csr(A)
-        M.reorder(sr.default_params(**_plan_kw(16, 1, 0), world=world, rank=r))
+        M.reorder(sr.default_params(**_plan_kw(panel, 1, 0), world=world, rank=r))
         st = M.stats()
         Cr = M.spmm(B)
         outr = M.sddmm(X, Y)
@@ -305,8 +309,8 @@ def test_shard_simulation(env, oracle, world):
         C[rows] = Cr.cpu().numpy()
         out[M.shard_nnz_ids()] = outr.cpu().numpy()
         if ref_cuts is None:
-            ref = oracle.plan(A, **_plan_kw(16, 1, 0))
-            P = 16
+            ref = oracle.plan(A, **_plan_kw(panel, 1, 0))
+            P = panel
             w = [int(ref["drow_ptr"][min(500, (p + 1) * P)] - ref["drow_ptr"][p * P]
                      + ref["rrow_ptr"][min(500, (p + 1) * P)] - ref["rrow_ptr"][p * P]) for p in range(ref["npanels"])]
             ref_cuts = oracle.partition(np.array(w), world)
@@ -578,7 +582,7 @@ def test_set_values_reuses_the_plan(env, oracle):
     sr, torch = env
     A = g.random_csr(700, 500, 0.03, 5, empty_frac=0.1)
     A2 = g.CSR(A.nrows, A.ncols, A.rowptr, A.colidx, g._uniform_vals(A.nnz, 77))
-    for params in (None, sr.default_params(**_plan_kw(16, 1, 8), tile_cols=8)):
+    for params in (None, sr.default_params(**_plan_kw(16, 1, 8), tile_cols=8), sr.default_params(**_plan_kw(8, 1, 8))):
         M = sr.SparseMatrix.from_csr(A)
         if params is not None:
             M.reorder(params)
