@@ -20,6 +20,27 @@ namespace sr {
 static thread_local std::string g_err;
 void set_error(const std::string& msg) { g_err = msg; }
 
+void keep_pool_memory() {
+  static int done = [] {
+    int dev = 0;
+    cudaMemPool_t pool;
+    if (cudaGetDevice(&dev) == cudaSuccess && cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+      uint64_t thr = ~0ull;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    cudaGetLastError();
+    return 1;
+  }();
+  (void)done;
+}
+
+static void trim_pool(int device) {
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) cudaMemPoolTrimTo(pool, 0);
+  cudaGetLastError();
+}
+
+
 namespace {
 
 constexpr int32_t kSplitChunk = 256;  // phase-S work item: at most this many nnz
@@ -235,23 +256,33 @@ int build_rt_stream(sr_csr_s* h, int64_t pb, int64_t pe, const std::vector<int32
   std::vector<int32_t> oidx;
   std::vector<int4> units;
   std::vector<std::array<int32_t, 3>> cell;  // (slot, row, dense nnz index)
+  std::vector<int2> split;                   // per unit: {panel's first slot, chunk << 16 | chunks}
+  int64_t n_slots = 0;
   for (int64_t p = pb; p < pe; ++p) {
     const int64_t dc0 = T.dense_ptr[p], dc1 = T.dense_ptr[p + 1];
     if (dc1 == dc0) continue;
     const int64_t q0 = p * PR, nrows = std::min<int64_t>(M, q0 + PR) - q0;
-    if (T.drow_ptr[q0 + nrows] - T.drow_ptr[q0] > kRtMaxPanelEntries) continue;  // TMA engine
     cell.clear();
     for (int64_t r = 0; r < nrows; ++r)
       for (int64_t e = T.drow_ptr[q0 + r]; e < T.drow_ptr[q0 + r + 1]; ++e)
         cell.push_back({T.d_slot[e], (int32_t)r, (int32_t)e});
     std::sort(cell.begin(), cell.end());
-    const int64_t e0 = (int64_t)ent.size();
+    // a panel with more than kRtChunk entries is cut at column boundaries into chunks, one warp
+    // each; SpMM chunks leave partial sums and the last one adds them in chunk order
+    int64_t e0 = (int64_t)ent.size();
+    const size_t first_unit = units.size();
     size_t i = 0;
     while (i < cell.size()) {
       size_t j = i;
       uint32_t mask = 0;
       while (j < cell.size() && cell[j][0] == cell[i][0]) mask |= 1u << cell[j++][1];
-      const int64_t len = 1 + (int64_t)(j - i), at = ((int64_t)ent.size() - e0) % 32;
+      const int64_t len = 1 + (int64_t)(j - i);
+      int64_t at = ((int64_t)ent.size() - e0) % 32;
+      if ((int64_t)ent.size() - e0 + (at + len > 32 ? 32 - at : 0) + len > kRtChunk) {  // close the chunk
+        units.push_back(make_int4((int32_t)e0, (int32_t)ent.size(), (int32_t)q0, (int32_t)nrows));
+        e0 = (int64_t)ent.size();
+        at = 0;
+      }
       if (at + len > 32)  // keep the column inside one 32-entry batch
         for (int64_t k = at; k < 32; ++k) {
           ent.push_back(make_int2(0, 0));
@@ -267,11 +298,35 @@ int build_rt_stream(sr_csr_s* h, int64_t pb, int64_t pe, const std::vector<int32
       i = j;
     }
     units.push_back(make_int4((int32_t)e0, (int32_t)ent.size(), (int32_t)q0, (int32_t)nrows));
+    const int32_t nch = (int32_t)(units.size() - first_unit);
+    for (int32_t c = 0; c < nch; ++c)
+      split.push_back(nch > 1 ? make_int2((int32_t)n_slots, (c << 16) | nch) : make_int2(-1, 1));
+    if (nch > 1) n_slots += nch;
   }
-  std::stable_sort(units.begin(), units.end(), [](const int4& a, const int4& b) { return a.y - a.x > b.y - b.x; });
+  {  // largest first (balance); the split records travel with their units
+    std::vector<size_t> ord(units.size());
+    std::iota(ord.begin(), ord.end(), 0);
+    std::stable_sort(ord.begin(), ord.end(), [&](size_t x, size_t y) {
+      return units[x].y - units[x].x > units[y].y - units[y].x;
+    });
+    std::vector<int4> u2(units.size());
+    std::vector<int2> s2(units.size());
+    for (size_t k = 0; k < ord.size(); ++k) {
+      u2[k] = units[ord[k]];
+      s2[k] = split[ord[k]];
+    }
+    units.swap(u2);
+    split.swap(s2);
+  }
   ent.resize(ent.size() + kEntPad, make_int2(0, 0));
   oidx.resize(oidx.size() + kEntPad, -1);
   P.n_rt = (int64_t)units.size();
+  P.n_rt_slots = n_slots;
+  SR_TRY(P.rt_split.upload(split, s));
+  if (n_slots > 0) {
+    SR_TRY(P.rt_counter.alloc((size_t)n_slots));
+    SR_CUDA_TRY(cudaMemsetAsync(P.rt_counter.p, 0, n_slots * sizeof(int32_t), s));
+  }
   SR_TRY(P.rt_units.upload(units, s));
   SR_TRY(P.rt_ent.upload(ent, s));
   SR_TRY(P.rt_oidx.upload(oidx, s));
@@ -379,14 +434,11 @@ int build_exec_plan_into(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s, De
     }
   };
   // panels of <= kRtMaxRows rows run on the register-tile engine (build_rt_stream) instead
-  // except panels with more than kRtMaxPanelEntries dense nnz (hub rows: one warp would serialise
-  // them), which stay on this engine with its split units and ordered combine
   const bool rt = PR <= kRtMaxRows;
-  for (int64_t p = pb; p < pe; ++p) {
+  for (int64_t p = pb; p < pe && !rt; ++p) {
     const int64_t dc0 = T.dense_ptr[p], dc1 = T.dense_ptr[p + 1];
     if (dc1 == dc0) continue;
     const int64_t q0 = p * PR, nrows = std::min<int64_t>(M, q0 + PR) - q0;
-    if (rt && T.drow_ptr[q0 + nrows] - T.drow_ptr[q0] <= kRtMaxPanelEntries) continue;
     const int64_t nd = dc1 - dc0, nt = (nd + TW - 1) / TW;
     maxd = std::max(maxd, nd);
     for (int64_t r = 0; r < nrows; ++r) cur[r] = T.drow_ptr[q0 + r];
@@ -550,8 +602,6 @@ int build_exec_plan_into(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s, De
     }
     if (rt) {  // register tiles: every dense column of a panel is gathered once per K pass
       for (int64_t p = pb; p < pe; ++p) {
-        const int64_t q0 = p * PR, q1 = std::min<int64_t>(M, q0 + PR);
-        if (T.drow_ptr[q1] - T.drow_ptr[q0] > kRtMaxPanelEntries) continue;  // counted with the vtiles
         for (int64_t k = T.dense_ptr[p]; k < T.dense_ptr[p + 1]; ++k) {
           ++tm.dense_col_loads;
           if (!seen[T.dense_cols[k]]) {
@@ -811,7 +861,6 @@ int sr_reorder(sr_csr h, const sr_reorder_params* p, sr_stream stream) {
   Tiling t_id;
   tile_rows(A, ident, p->panel_rows, dense_min0, t_id);
   st.dense0 = t_id.n_dense();
-  if (dense_min0 != p->dense_min) tile_rows(A, ident, p->panel_rows, p->dense_min, t_id);
   st.t_tile_s += now_s() - t0;
   bool round1 = p->mode == SR_REORDER_FORCE;
   if (p->mode == SR_REORDER_AUTO)
@@ -825,6 +874,11 @@ int sr_reorder(sr_csr h, const sr_reorder_params* p, sr_stream stream) {
     st.t_tile_s += now_s() - t0;
   } else {
     h->perm1 = ident;
+    if (dense_min0 != p->dense_min) {  // the plan tiles with the execution threshold
+      t0 = now_s();
+      tile_rows(A, ident, p->panel_rows, p->dense_min, t_id);
+      st.t_tile_s += now_s() - t0;
+    }
     h->tiles = std::move(t_id);
   }
   st.round1 = round1 ? 1 : 0;
@@ -852,6 +906,8 @@ int sr_reorder(sr_csr h, const sr_reorder_params* p, sr_stream stream) {
     if (T.rrow_ptr[q + 1] > T.rrow_ptr[q]) h->perm2.push_back(q);
   st.n_perm2 = (int64_t)h->perm2.size();
   SR_TRY(finish_plan(h, s));
+  cudaStreamSynchronize(s);
+  trim_pool(h->device);  // give back the LSH rounds' pooled temporaries
   st.t_total_s = now_s() - t_start;
   rollback.commit();
   return SR_OK;

@@ -374,10 +374,10 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
   while (init_pos > 0 && init[init_pos - 1].inter == 0) --init_pos;
   size_t cur = 0, zc = 0;
   int64_t nclusters = M;
-  // roots changed by a merge since the current block's speculative evaluation: a 4096-bit
+  // roots changed by a merge since the current block's speculative evaluation: a 2^16-bit
   // filter (false positives only send a pop down the sequential path)
-  uint64_t modbits[64];
-  auto mod_bit = [](int32_t x) { return (uint32_t)((uint32_t)x * 0x9E3779B1u) >> 20; };
+  uint64_t modbits[1024];
+  auto mod_bit = [](int32_t x) { return (uint32_t)((uint32_t)x * 0x9E3779B1u) >> 16; };
   auto mark_mod = [&](int32_t x) { const uint32_t b = mod_bit(x); modbits[b >> 6] |= 1ull << (b & 63); };
   auto is_mod = [&](int32_t x) { const uint32_t b = mod_bit(x); return (modbits[b >> 6] >> (b & 63)) & 1ull; };
   std::memset(modbits, 0, sizeof(modbits));
@@ -444,7 +444,11 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
     uint32_t inter, uni;
     int32_t cls;
   };
-  constexpr size_t BS = 4096;
+  static const size_t BS = [] {  // block size of the speculative pass (SR_CLUSTER_BS, measurement knob)
+    const char* e = getenv("SR_CLUSTER_BS");
+    const long v = e ? atol(e) : 8192;
+    return (size_t)(v < 64 ? 64 : v);
+  }();
   std::vector<Pre> pre(BS);
   size_t blk0 = 0, blk1 = 0;
   int64_t n_spec_used = 0;
@@ -452,7 +456,9 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
     while (nd[x].parent != x) x = nd[x].parent;
     return x;
   };
+  double t_eval = 0.0;
   auto evaluate_block = [&](size_t from) {
+    const double te = dbg ? now() : 0.0;
     flush_recent();  // the speculative pass reads `members` only
     midflush = false;
     blk0 = from;
@@ -484,6 +490,7 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
       p.uni = c.uni;
       p.cls = 3;
     }
+    if (dbg) t_eval += now() - te;
   };
   constexpr size_t PF = 32, PF2 = 16, PF3 = 8;  // prefetch distances (sequential mode)
   while (nclusters > 0) {
@@ -553,8 +560,8 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
       } else {
         zero_phase = true;
         if (dbg)
-          fprintf(stderr, "  J>0 phase %.3f s, %lld clusters left, %zu J=0 pairs, %lld speculative results used\n",
-                  now() - t2, (long long)nclusters, zero_keys.size(), (long long)n_spec_used);
+          fprintf(stderr, "  J>0 phase %.3f s (speculative blocks %.3f s), %lld clusters left, %zu J=0 pairs, %lld speculative results used\n",
+                  now() - t2, t_eval, (long long)nclusters, zero_keys.size(), (long long)n_spec_used);
         for (size_t e = init_pos; e < (size_t)npairs; ++e) zero_keys.push_back(((uint64_t)init[e].i << 32) | init[e].j);
         __gnu_parallel::sort(zero_keys.begin(), zero_keys.end());
         continue;

@@ -559,7 +559,8 @@ template <int U, int VEC, int MINB>
 __global__ void __launch_bounds__(256, MINB) spmm_rtile_kernel(
     const int4* __restrict__ units, int64_t n_units, const int2* __restrict__ ent,
     const int32_t* __restrict__ dense_out, const float* __restrict__ B, uint32_t ldb, float* __restrict__ C,
-    int64_t ldc, int kw) {
+    int64_t ldc, int kw, const int2* __restrict__ split, float* __restrict__ scratch, int* __restrict__ counter,
+    int K, int k0) {
   constexpr int P = kRtMaxRows;
   const int lane = threadIdx.x & 31;
   const int64_t w = (int64_t)blockIdx.x * (blockDim.x >> 5) + __shfl_sync(FULL, threadIdx.x >> 5, 0);
@@ -605,6 +606,33 @@ __global__ void __launch_bounds__(256, MINB) spmm_rtile_kernel(
     }
   }
   const int orow = lane < u.w ? __ldg(dense_out + u.z + lane) : -1;
+  const int2 sp = __ldg(split + w);
+  if (sp.x >= 0) {  // one chunk of a hub panel: partials -> scratch; the last chunk adds them in order
+    const int c = sp.y >> 16, nch = sp.y & 0xffff;
+    float* sc = scratch + (int64_t)(sp.x + c) * P * K + k0 + lane * VEC;
+#pragma unroll
+    for (int r = 0; r < P; ++r)
+      if (kv) acc[r].store(sc + (int64_t)r * K);
+    __threadfence();
+    __syncwarp();
+    int last = 0;
+    if (lane == 0) last = (atomicAdd(counter + sp.x, 1) == nch - 1);
+    last = __shfl_sync(FULL, last, 0);
+    if (!last) return;
+    __threadfence();
+#pragma unroll
+    for (int r = 0; r < P; ++r) acc[r].zero();
+    for (int cc = 0; cc < nch; ++cc) {
+      const float* src = scratch + (int64_t)(sp.x + cc) * P * K + k0 + lane * VEC;
+#pragma unroll
+      for (int r = 0; r < P; ++r) {
+        Frag<VEC> part;
+        if (kv) part.load_cg(src + (int64_t)r * K); else part.zero();
+        acc[r].add(part);
+      }
+    }
+    if (lane == 0) counter[sp.x] = 0;
+  }
 #pragma unroll
   for (int r = 0; r < P; ++r) {
     const int o = __shfl_sync(FULL, orow, r);
@@ -1214,10 +1242,6 @@ int env_int(const char* name, int dflt) {
   const char* d = getenv(name);
   return d ? atoi(d) : dflt;
 }
-int rt_variant() {  // SR_RT_VARIANT (measurement knob): register-tile SpMM lane width / columns in flight
-  static const int v = env_int("SR_RT_VARIANT", 0);
-  return v;
-}
 bool task_kernels() {
   static const bool v = env_int("SR_PHASE_S", 1) != 0;
   return v;
@@ -1244,23 +1268,21 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
   if (P.n_rt > 0) {  // register-tile phase D (panels of <= kRtMaxRows rows)
     const unsigned grid = (unsigned)((P.n_rt + kSparseWarps - 1) / kSparseWarps);
     if (P.profiling) SR_TRY(prof_begin(P, 5, s));
-    const int rv = rt_variant();
+    if (P.n_rt_slots > 0 && P.rt_scratch_k < K) {
+      SR_TRY(P.rt_scratch.alloc((size_t)P.n_rt_slots * kRtMaxRows * K));
+      P.rt_scratch_k = K;
+    }
     auto rk = [&](auto kern, int vec) {
       const int pass = 32 * vec;
       for (int64_t k0 = 0; k0 < K; k0 += pass)
         kern<<<grid, kSparseWarps * 32, 0, s>>>(P.rt_units.p, P.n_rt, P.rt_ent.p, P.dense_out.p, B + k0,
-                                                 (uint32_t)(ldb * 4), C + k0, ldc, (int)std::min<int64_t>(pass, K - k0));
+                                                 (uint32_t)(ldb * 4), C + k0, ldc, (int)std::min<int64_t>(pass, K - k0),
+                                                 P.rt_split.p, P.rt_scratch.p, P.rt_counter.p, (int)K, (int)k0);
     };
-    if constexpr (VEC == 4) {
-      switch (rv) {
-        case 1: rk(spmm_rtile_kernel<8, 4, 3>, 4); break;
-        case 2: rk(spmm_rtile_kernel<8, 2, 6>, 2); break;
-        case 3: rk(spmm_rtile_kernel<4, 2, 8>, 2); break;
-        default: rk(spmm_rtile_kernel<4, 4, 4>, 4); break;
-      }
-    } else {
+    if constexpr (VEC == 4)
+      rk(spmm_rtile_kernel<4, 4, 4>, 4);  // 4 columns in flight, 64 registers (profiles/r02 session f-h)
+    else
       rk(spmm_rtile_kernel<8, 1, 8>, 1);
-    }
     SR_CUDA_TRY(cudaGetLastError());
     if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;

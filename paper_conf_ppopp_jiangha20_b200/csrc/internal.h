@@ -34,19 +34,27 @@ struct Status {
   } while (0)
 
 // RAII device buffer
+// Stream-ordered pool allocations (cudaMallocAsync) for the reorder's temporaries: the two LSH
+// rounds allocate and free GBs of sort buffers; the device's default pool keeps them mapped
+// between rounds instead of a cudaMalloc / cudaFree of each (sr_reorder trims it at the end).
+void keep_pool_memory();
+
 template <typename T>
 struct DevBuf {
   T* p = nullptr;
   size_t n = 0;
+  cudaStream_t pool = nullptr;  // non-null: stream-ordered allocation on this stream
   DevBuf() = default;
+  explicit DevBuf(cudaStream_t s) : pool(s) { keep_pool_memory(); }
   DevBuf(const DevBuf&) = delete;
   DevBuf& operator=(const DevBuf&) = delete;
-  DevBuf(DevBuf&& o) noexcept : p(o.p), n(o.n) { o.p = nullptr; o.n = 0; }
+  DevBuf(DevBuf&& o) noexcept : p(o.p), n(o.n), pool(o.pool) { o.p = nullptr; o.n = 0; }
   DevBuf& operator=(DevBuf&& o) noexcept {
     if (this != &o) {
       release();
       p = o.p;
       n = o.n;
+      pool = o.pool;
       o.p = nullptr;
       o.n = 0;
     }
@@ -54,14 +62,21 @@ struct DevBuf {
   }
   ~DevBuf() { release(); }
   void release() {
-    if (p) cudaFree(p);
+    if (p) {
+      if (pool)
+        cudaFreeAsync(p, pool);
+      else
+        cudaFree(p);
+    }
     p = nullptr;
     n = 0;
   }
   int alloc(size_t count) {
     release();
     if (count == 0) count = 1;
-    if (cudaMalloc(&p, count * sizeof(T)) != cudaSuccess) {
+    const cudaError_t e = pool ? cudaMallocAsync(reinterpret_cast<void**>(&p), count * sizeof(T), pool)
+                               : cudaMalloc(&p, count * sizeof(T));
+    if (e != cudaSuccess) {
       cudaGetLastError();
       set_error("cudaMalloc of " + std::to_string(count * sizeof(T)) + " bytes failed");
       p = nullptr;
@@ -135,7 +150,7 @@ struct __align__(16) DUnit {
   int32_t pad0, pad1, pad2;
 };
 constexpr int kRtMaxRows = 8;                        // register-tile engine: panel rows
-constexpr int64_t kRtMaxPanelEntries = 4096;         // larger panels stay on the TMA engine
+constexpr int64_t kRtChunk = 1024;                   // register-tile stream entries per warp (chunk)
 constexpr int32_t kRtHeader = (int32_t)0x80000000u;  // marks a column header entry
 constexpr int kMaxUnitTiles = 8;
 constexpr int kMaxExecTile = 64;
@@ -180,6 +195,11 @@ struct DevPlan {
   DevBuf<int4> rt_units;      // one warp per panel: {e0, e1, first position, rows}
   DevBuf<int2> rt_ent;        // column headers {col | kRtHeader, row mask} + {row, value bits}
   DevBuf<int32_t> rt_oidx;    // SDDMM output index per value entry (-1: header / padding)
+  DevBuf<int2> rt_split;      // per unit: {panel's first slot, chunk << 16 | chunks} ({-1, 1}: whole panel)
+  DevBuf<int32_t> rt_counter; // per split panel (its first slot): finished chunks
+  int64_t n_rt_slots = 0;
+  DevBuf<float> rt_scratch;   // n_rt_slots × kRtMaxRows × rt_scratch_k partial sums
+  int64_t rt_scratch_k = 0;
   DevBuf<int32_t> pos_xrow;   // position -> original row
   DevBuf<int32_t> pos_out;    // position -> SpMM output row
   DevBuf<int32_t> dense_out;  // position -> SpMM output row if the row has dense nnz, else -1

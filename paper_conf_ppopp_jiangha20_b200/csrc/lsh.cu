@@ -298,16 +298,16 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
     ha[t] = (uint32_t)(next_splitmix(st) & 0xFFFFFFFFull) | 1u;
     hb[t] = (uint32_t)(next_splitmix(st) & 0xFFFFFFFFull);
   }
-  DevBuf<int64_t> d_rowptr;
-  DevBuf<int32_t> d_col, d_live;
-  DevBuf<uint32_t> d_a, d_b;
+  DevBuf<int64_t> d_rowptr(s);
+  DevBuf<int32_t> d_col(s), d_live(s);
+  DevBuf<uint32_t> d_a(s), d_b(s);
   SR_TRY(d_rowptr.upload(rowptr_h, (size_t)M + 1, s));
   SR_TRY(d_col.upload(col_h, (size_t)nnz, s));
   SR_TRY(d_live.upload(live, s));
   SR_TRY(d_a.upload(ha, s));
   SR_TRY(d_b.upload(hb, s));
   lap("host prep + uploads");
-  DevBuf<uint64_t> keys;
+  DevBuf<uint64_t> keys(s);
   SR_TRY(keys.alloc((size_t)nb * L));
   {
     const int threads = 256;
@@ -325,10 +325,10 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
   }
   lap("minhash");
   // per band: sort, bucket, emit
-  DevBuf<uint64_t> kout;
-  DevBuf<int32_t> vin, vout, run_len, run_of, nruns_d;
-  DevBuf<uint64_t> run_key;
-  DevBuf<int64_t> run_start, run_npairs, run_off;
+  DevBuf<uint64_t> kout(s);
+  DevBuf<int32_t> vin(s), vout(s), run_len(s), run_of(s), nruns_d(s);
+  DevBuf<uint64_t> run_key(s);
+  DevBuf<int64_t> run_start(s), run_npairs(s), run_off(s);
   SR_TRY(kout.alloc(L));
   SR_TRY(vin.alloc(L));
   SR_TRY(vout.alloc(L));
@@ -345,7 +345,7 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
     SR_CUDA_TRY(cudaMemcpyAsync(vin.p, iota.data(), L * sizeof(int32_t), cudaMemcpyHostToDevice, s));
     SR_CUDA_TRY(cudaStreamSynchronize(s));
   }
-  DevBuf<uint8_t> temp;
+  DevBuf<uint8_t> temp(s);
   size_t temp_bytes = 0;
   auto ensure_temp = [&](size_t need) -> int {
     if (need > temp_bytes) {
@@ -354,7 +354,7 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
     }
     return SR_OK;
   };
-  DevBuf<uint64_t> allpairs;
+  DevBuf<uint64_t> allpairs(s);
   int64_t cap_pairs = 0, n_pairs = 0;
   const int64_t C = p.max_bucket;
   for (int band = 0; band < nb; ++band) {
@@ -396,7 +396,7 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
     if (n_pairs + band_pairs > cap_pairs) {
       int64_t ncap = std::max<int64_t>(2 * cap_pairs, n_pairs + band_pairs);
       ncap = std::max<int64_t>(ncap, 1 << 20);
-      DevBuf<uint64_t> bigger;
+      DevBuf<uint64_t> bigger(s);
       SR_TRY(bigger.alloc(ncap));
       if (n_pairs)
         SR_CUDA_TRY(cudaMemcpyAsync(bigger.p, allpairs.p, n_pairs * sizeof(uint64_t),
@@ -416,8 +416,8 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
   keys.release();
   if (n_pairs == 0) return SR_OK;
   // union over bands: sort + unique
-  DevBuf<uint64_t> sorted, uniq;
-  DevBuf<int64_t> nuniq;
+  DevBuf<uint64_t> sorted(s), uniq(s);
+  DevBuf<int64_t> nuniq(s);
   SR_TRY(sorted.alloc(n_pairs));
   {
     size_t need = 0;
@@ -444,16 +444,16 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
     SR_CUDA_TRY(cudaMemcpyAsync(pairs_by_key->data(), allpairs.p, E * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
   }
   // exact Jaccard + heap-order sort
-  DevBuf<uint32_t> d_inter, d_uni, idx_in, idx_out, i2, u2;
-  DevBuf<uint64_t> jkey, jkey_out, p2;
+  DevBuf<uint32_t> d_inter(s), d_uni(s), idx_in(s), idx_out(s), i2(s), u2(s);
+  DevBuf<uint64_t> jkey(s), jkey_out(s), p2(s);
   SR_TRY(d_inter.alloc(E));
   SR_TRY(d_uni.alloc(E));
   SR_TRY(jkey.alloc(E));
   SR_TRY(jkey_out.alloc(E));
   SR_TRY(idx_in.alloc(E));
   SR_TRY(idx_out.alloc(E));
-  DevBuf<int64_t> long_idx;
-  DevBuf<int> n_long;
+  DevBuf<int64_t> long_idx(s);
+  DevBuf<int> n_long(s);
   SR_TRY(long_idx.alloc(E));
   SR_TRY(n_long.alloc(1));
   SR_CUDA_TRY(cudaMemsetAsync(n_long.p, 0, sizeof(int), s));

@@ -59,6 +59,7 @@ def main():
     run(tiny, sr.default_params(**dict(force, panel_rows=8)), (32, 36, 128, 132))  # register-tile phase D
     H = matrix_with_long_rows_and_hub()
     M = run(H, sr.default_params(**force), (32, 128, 256))
+    run(H, sr.default_params(**dict(force, panel_rows=8, mode=sr.OFF)), (32, 128, 256))  # split register tiles
     st = M.stats()
     assert st["dense1"] > 0 and st["ntiles"] > 8, st
     # new values on the same plan

@@ -33,6 +33,15 @@ def test_exports_every_declared_symbol(sr):
     assert declared == set(sr.EXPORTED)
 
 
+def test_no_unresolved_library_symbols(sr):
+    """Every symbol of the library's own namespace is defined inside libsr.so (a declaration
+    without a definition would only fail when the library is loaded on the GPU box)."""
+    import subprocess
+    out = subprocess.check_output(["nm", "-D", "--undefined-only", sr.LIB_PATH], text=True)
+    missing = [l for l in out.splitlines() if "_ZN2sr" in l or " sr_" in l]
+    assert not missing, missing
+
+
 def _c_layout(struct, fields):
     """sizeof / offsetof of a struct of include/sr.h, compiled with gcc (the header is the
     authority the ctypes binding must match)."""

@@ -179,6 +179,33 @@ def test_long_rows_split_and_rmw(env, oracle):
             np.testing.assert_array_equal(C, C2)
 
 
+@pytest.mark.parametrize("K", [32, 128, 256])
+def test_register_tiles_split_hub_panels(env, oracle, K):
+    """Panels of 8 rows on the register-tile engine where one panel holds thousands of dense
+    entries: it is cut into chunks (one warp each) whose partial sums the last chunk adds in
+    chunk order; the result is deterministic and matches the oracle."""
+    sr, torch = env
+    rng = np.random.default_rng(3)
+    n, m = 64, 6000
+    rows, cols = [], []
+    for i in range(n):
+        d = int(rng.integers(1, 30))
+        rows.append(np.full(d, i))
+        cols.append(rng.choice(m, size=d, replace=False))
+    for i in range(8, 16):  # panel 1: 8 rows sharing 2500 columns -> ~22 k entries, ~22 chunks
+        rows.append(np.full(2500, i))
+        cols.append(np.arange(3000, 5500))
+    rowptr, colidx = g._from_coo(n, m, np.concatenate(rows), np.concatenate(cols))
+    A = g.CSR(n, m, rowptr, colidx, g._uniform_vals(colidx.size, 5))
+    params = sr.default_params(**_plan_kw(8, 2, 0))  # OFF: identity order, tiles only
+    M, B, X, Y, C, out = _run(env, A, K, params)
+    assert M.stats()["dense1"] >= 8 * 2500
+    _spmm_check(oracle, A, B, C)
+    _sddmm_check(oracle, A, X, Y, out)
+    _, _, _, _, C2, _ = _run(env, A, K, params)
+    np.testing.assert_array_equal(C, C2)
+
+
 def test_unsorted_input_keeps_caller_nnz_order(env, oracle):
     sr, _ = env
     A = g.random_csr(120, 90, 0.1, 12, empty_frac=0.1)
