@@ -57,7 +57,7 @@ def parse(argv=None):
     ap.add_argument("--config", default="rmat", choices=list(gen.CONFIGS))
     ap.add_argument("--K", type=int, default=128)
     ap.add_argument("--extra-K", default=None,
-                    help="comma list of further K timed on the same plan (default: 32 for rmat at K=128)")
+                    help="comma list of further K timed on the same plan (default: 32 for rmat at K=128; 'none')")
     ap.add_argument("--ops", default="spmm,sddmm")
     ap.add_argument("--mode", default="auto", choices=["auto", "force", "off"])
     ap.add_argument("--panel-rows", type=int, default=64)
@@ -567,6 +567,7 @@ def run_ours(args, A, ops, rank, world, local_rank):
     # further K on the same plan (BASELINE metric: K = 32 and 128)
     extra = {}
     ks = args.extra_K if args.extra_K is not None else ("32" if args.config == "rmat" and K == 128 else "")
+    ks = "" if ks == "none" else ks
     for k2 in [int(x) for x in ks.split(",") if x.strip()]:
         S2 = Stepper(torch, M, A, k2, ops, dev, flush, stream)
         for _ in range(max(3, args.warmup)):
