@@ -714,7 +714,7 @@ def run_ours(args, A, ops, rank, world, local_rank):
             "extra_K": extra,
             "preprocess": {"seconds": t_pre, "lsh1_s": stp["t_lsh1_s"], "cluster1_s": stp["t_cluster1_s"],
                            "tile_s": stp["t_tile_s"], "lsh2_s": stp["t_lsh2_s"], "cluster2_s": stp["t_cluster2_s"],
-                           "plan_build_s": stp["t_plan_s"],
+                           "plan_build_s": stp["t_plan_s"], "reorder_call_s": stp["t_total_s"],
                            "round1": stp["round1"], "round2": stp["round2"], "E1": stp["E1"], "E2": stp["E2"],
                            "dense_ratio0": stp["dense0"] / max(1, stp["nnz"]),
                            "dense_ratio": stp["dense1"] / max(1, stp["nnz"]),

@@ -3,6 +3,7 @@
 #include <algorithm>
 #include <array>
 #include <chrono>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <numeric>
@@ -905,10 +906,18 @@ int sr_reorder(sr_csr h, const sr_reorder_params* p, sr_stream stream) {
   for (int32_t q : order)
     if (T.rrow_ptr[q + 1] > T.rrow_ptr[q]) h->perm2.push_back(q);
   st.n_perm2 = (int64_t)h->perm2.size();
+  const double t_fin = now_s();
   SR_TRY(finish_plan(h, s));
+  const double t_trim = now_s();
   cudaStreamSynchronize(s);
-  trim_pool(h->device);  // give back the LSH rounds' pooled temporaries
+  if (!getenv("SR_POOL_KEEP")) trim_pool(h->device);  // give back the LSH rounds' pooled temporaries
   st.t_total_s = now_s() - t_start;
+  if (getenv("SR_DEBUG_REORDER"))
+    fprintf(stderr, "sr_reorder: total %.3f s = lsh %.3f + %.3f, cluster %.3f + %.3f, tile %.3f, finish_plan %.3f "
+            "(exec plan %.3f), trim %.3f, other %.3f\n", st.t_total_s, st.t_lsh1_s, st.t_lsh2_s, st.t_cluster1_s,
+            st.t_cluster2_s, st.t_tile_s, t_trim - t_fin, st.t_plan_s, now_s() - t_trim,
+            st.t_total_s - (st.t_lsh1_s + st.t_lsh2_s + st.t_cluster1_s + st.t_cluster2_s + st.t_tile_s +
+                            (now_s() - t_fin)));
   rollback.commit();
   return SR_OK;
 }

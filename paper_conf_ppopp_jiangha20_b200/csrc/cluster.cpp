@@ -20,6 +20,7 @@
 //  SR_DEBUG_CLUSTER=1 prints the phase times.
 // Readings R3-R12 decide everything the paper leaves open.
 #include <algorithm>
+#include <atomic>
 #include <chrono>
 #include <cstdio>
 #include <cstdlib>
@@ -29,6 +30,10 @@
 #include <memory>
 #include <numeric>
 #include <vector>
+
+#ifdef _OPENMP
+#include <omp.h>
+#endif
 
 #include "internal.h"
 
@@ -100,10 +105,10 @@ class PairSet {
     reset(cap);
   }
   void prefetch(uint64_t k) const { __builtin_prefetch(&slots_[hash(k) & mask_]); }
-  bool contains(uint64_t k) const {
+  bool contains(uint64_t k) const {  // relaxed atomic loads: may run beside concurrent CAS inserts
     size_t h = hash(k) & mask_;
     while (true) {
-      const uint64_t v = slots_[h];
+      const uint64_t v = __atomic_load_n(&slots_[h], __ATOMIC_RELAXED);
       if (v == k) return true;
       if (v == kEmpty) return false;
       h = (h + 1) & mask_;
@@ -198,9 +203,9 @@ class SmallSet {
   }
 
  private:
-  static constexpr size_t kCap = 1 << 14;
+  static constexpr size_t kCap = 1 << 16;
   static constexpr uint64_t kEmpty = ~0ull;
-  static size_t mix(uint64_t k) { return (size_t)((k * 0x9E3779B97F4A7C15ull) >> 50) & (kCap - 1); }
+  static size_t mix(uint64_t k) { return (size_t)((k * 0x9E3779B97F4A7C15ull) >> 48) & (kCap - 1); }
   std::vector<uint64_t> slots_;
   std::vector<uint32_t> used_;
   std::vector<uint64_t> keys_;
@@ -337,9 +342,13 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
 
   std::vector<Node> nd((size_t)M);
   for (int64_t x = 0; x < M; ++x) nd[x] = Node{(int32_t)x, 1u};
+  // The union-find nodes are written only by the thread running Alg 3; the pipelined speculative
+  // pass reads them concurrently, so the writes are relaxed atomic stores (plain moves on x86).
+  auto set_parent = [&](int32_t x, int32_t v) { __atomic_store_n(&nd[x].parent, v, __ATOMIC_RELAXED); };
+  auto set_size = [&](int32_t x, uint32_t v) { __atomic_store_n(&nd[x].sz, v, __ATOMIC_RELAXED); };
   auto root = [&](int32_t x) {  // path halving
     while (x != nd[x].parent) {
-      nd[x].parent = nd[nd[x].parent].parent;
+      set_parent(x, nd[nd[x].parent].parent);
       x = nd[x].parent;
     }
     return x;
@@ -406,11 +415,11 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
       // the larger cluster absorbs the smaller; equal sizes: smaller index (R6)
       const bool i_wins = nd[i].sz > nd[j].sz || (nd[i].sz == nd[j].sz && i < j);
       const int32_t w = i_wins ? i : j, l = i_wins ? j : i;
-      nd[l].parent = w;
-      nd[w].sz += nd[l].sz;  // R4
+      set_parent(l, w);
+      set_size(w, nd[w].sz + nd[l].sz);  // R4
       --nclusters;
       if (nd[w].sz >= (uint32_t)threshold_size) {  // R7, R5
-        nd[w].sz |= kDeleted;
+        set_size(w, nd[w].sz | kDeleted);
         --nclusters;
       }
       mark_mod(w);
@@ -492,6 +501,234 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
     }
     if (dbg) t_eval += now() - te;
   };
+  // ---- Pipelined variant of the speculative pass (the default with >= 3 OpenMP threads): the
+  // evaluation of block b+1 runs on the other threads while this thread replays block b, so the
+  // replay (the sequential part) is the phase's critical path.  The evaluators read the union-find
+  // nodes while the replay writes them (relaxed atomics), so a block's results are checked against
+  // every merge since its evaluation began (the merged-root filters of the current and the previous
+  // block); skips because of equal or deleted roots stay valid under any interleaving (both facts
+  // are permanent, and an observed parent chain only ever leads to an ancestor).  Re-inserted pairs
+  // go to small per-block sets; the keys of block b-1 are added to the big set by the evaluators of
+  // block b+1 before they evaluate it, so a block's "not a candidate" results are re-checked against
+  // the sets of the previous and the current block only.
+  int nthr = 1;
+#ifdef _OPENMP
+  nthr = omp_get_max_threads();
+#endif
+  if (spec && nthr >= 3 && init_pos > 0 && getenv("SR_CLUSTER_NOPIPE") == nullptr) {
+    const int64_t nblocks = (int64_t)((init_pos + BS - 1) / BS);
+    std::vector<Pre> ring[2] = {std::vector<Pre>(BS), std::vector<Pre>(BS)};
+    SmallSet kset[2];  // keys re-inserted while replaying the previous / the current block
+    int kprev = 0, kcur = 1;
+    uint64_t fbits[2][1024];
+    std::memset(fbits, 0, sizeof(fbits));
+    int fprev = 0, fcur = 1;
+    auto fmark = [&](int32_t x) { const uint32_t b = mod_bit(x); fbits[fcur][b >> 6] |= 1ull << (b & 63); };
+    auto fmod = [&](int32_t x) {
+      const uint32_t b = mod_bit(x);
+      return ((fbits[fprev][b >> 6] | fbits[fcur][b >> 6]) >> (b & 63)) & 1ull;
+    };
+    bool overflow = false;  // a block's key set was flushed early: re-check class 3 against `members`
+    std::atomic<int64_t> req{-1}, ready{-1};
+    std::atomic<int64_t> flush_cur{0}, flush_done{0}, eval_cur{0}, eval_done{0};
+    std::atomic<bool> stop{false};
+    std::atomic<int> acks{0};  // evaluators done with the current request (all must be before the next)
+    const uint64_t* flush_keys = nullptr;
+    int64_t flush_n = 0, eval_b0 = 0, eval_len = 0;
+    Pre* eval_out = nullptr;
+    auto pause = [] { __builtin_ia32_pause(); };
+    auto cand_pipe = [&](uint64_t key) {
+      return kset[kcur].contains(key) || kset[kprev].contains(key) || is_candidate_big(key);
+    };
+    // replay-side versions of process()/reinsert() that use the per-block key sets and filters
+    auto reinsert_pipe = [&](const Cand& c, uint64_t key) {
+      if (kset[kcur].nearly_full()) {  // rare: flush it here (CAS inserts; the big set was reserved)
+        for (uint64_t k : kset[kcur].keys()) members.insert_distinct_concurrent(k);
+        members.set_size(members.size() + kset[kcur].keys().size());
+        kset[kcur].clear();
+        overflow = true;
+      }
+      kset[kcur].insert(key);
+      ++n_reinsert;
+      if (c.inter > 0) {
+        extra.push(c);
+      } else {
+        ++n_zero;
+        zero_keys.push_back(key);
+      }
+    };
+    auto process_pipe = [&](int32_t i, int32_t j) {
+      if (nd[i].parent == i && nd[j].parent == j) {
+        if ((nd[i].sz | nd[j].sz) & kDeleted) return;
+        const bool i_wins = nd[i].sz > nd[j].sz || (nd[i].sz == nd[j].sz && i < j);
+        const int32_t w = i_wins ? i : j, l = i_wins ? j : i;
+        set_parent(l, w);
+        set_size(w, nd[w].sz + nd[l].sz);  // R4
+        --nclusters;
+        if (nd[w].sz >= (uint32_t)threshold_size) {  // R7, R5
+          set_size(w, nd[w].sz | kDeleted);
+          --nclusters;
+        }
+        fmark(w);
+        fmark(l);
+      } else {
+        i = root(i);
+        j = root(j);
+        if (((nd[i].sz | nd[j].sz) & kDeleted) || i == j) return;
+        const uint32_t lo = (uint32_t)std::min(i, j), hi = (uint32_t)std::max(i, j);
+        const uint64_t key = ((uint64_t)lo << 32) | hi;
+        if (cand_pipe(key)) return;
+        Cand c;
+        similarity(lo, hi, &c);  // representing rows (R8)
+        reinsert_pipe(c, key);
+      }
+    };
+    auto evaluate_one = [&](int64_t k, Pre& p) {
+      const int32_t i = (int32_t)init[k].i, j = (int32_t)init[k].j;
+      const int32_t pi = __atomic_load_n(&nd[i].parent, __ATOMIC_RELAXED);
+      const int32_t pj = __atomic_load_n(&nd[j].parent, __ATOMIC_RELAXED);
+      if (pi == i && pj == j) {
+        p.cls = 0;
+        return;
+      }
+      int32_t ri = i, rj = j;
+      for (int32_t q; (q = __atomic_load_n(&nd[ri].parent, __ATOMIC_RELAXED)) != ri;) ri = q;
+      for (int32_t q; (q = __atomic_load_n(&nd[rj].parent, __ATOMIC_RELAXED)) != rj;) rj = q;
+      p.ri = ri;
+      p.rj = rj;
+      const uint32_t si = __atomic_load_n(&nd[ri].sz, __ATOMIC_RELAXED);
+      const uint32_t sj = __atomic_load_n(&nd[rj].sz, __ATOMIC_RELAXED);
+      if (((si | sj) & kDeleted) || ri == rj) {
+        p.cls = 1;
+        return;
+      }
+      const uint32_t lo = (uint32_t)std::min(ri, rj), hi = (uint32_t)std::max(ri, rj);
+      if (is_candidate_big(((uint64_t)lo << 32) | hi)) {
+        p.cls = 2;
+        return;
+      }
+      Cand c;
+      similarity(lo, hi, &c);
+      p.inter = c.inter;
+      p.uni = c.uni;
+      p.cls = 3;
+    };
+    // publish the next evaluation (the evaluators are idle: the previous one has completed)
+    auto request = [&](int64_t b, const std::vector<uint64_t>* keys) {
+      if (b > 0)  // every evaluator has left the previous request's loops
+        while (acks.load(std::memory_order_acquire) < nthr - 1) pause();
+      acks.store(0, std::memory_order_relaxed);
+      flush_n = keys ? (int64_t)keys->size() : 0;
+      members.reserve_more((size_t)flush_n + (size_t)BS * 4 + 65536);
+      members.set_size(members.size() + (size_t)flush_n);
+      flush_keys = keys ? keys->data() : nullptr;
+      eval_b0 = b * (int64_t)BS;
+      eval_len = std::min<int64_t>((int64_t)init_pos, eval_b0 + (int64_t)BS) - eval_b0;
+      eval_out = ring[b & 1].data();
+      flush_cur.store(0, std::memory_order_relaxed);
+      flush_done.store(0, std::memory_order_relaxed);
+      eval_cur.store(0, std::memory_order_relaxed);
+      eval_done.store(0, std::memory_order_relaxed);
+      req.store(b, std::memory_order_release);
+    };
+    auto wait_ready = [&](int64_t b) {
+      const double te = dbg ? now() : 0.0;
+      while (ready.load(std::memory_order_acquire) != b) pause();
+      if (dbg) t_eval += now() - te;  // time the replay waited for the evaluators
+    };
+#pragma omp parallel num_threads(nthr)
+    {
+      if (omp_get_thread_num() != 0) {  // evaluators
+        int64_t seen = -1;
+        while (true) {
+          int64_t r;
+          while ((r = req.load(std::memory_order_acquire)) == seen && !stop.load(std::memory_order_acquire)) pause();
+          if (r == seen) break;
+          seen = r;
+          for (;;) {
+            const int64_t k = flush_cur.fetch_add(512, std::memory_order_relaxed);
+            if (k >= flush_n) break;
+            const int64_t e = std::min(flush_n, k + 512);
+            for (int64_t t = k; t < e; ++t) members.insert_distinct_concurrent(flush_keys[t]);
+            flush_done.fetch_add(e - k, std::memory_order_release);
+          }
+          while (flush_done.load(std::memory_order_acquire) < flush_n) pause();
+          for (;;) {
+            const int64_t k = eval_cur.fetch_add(64, std::memory_order_relaxed);
+            if (k >= eval_len) break;
+            const int64_t e = std::min(eval_len, k + 64);
+            for (int64_t t = k; t < e; ++t) evaluate_one(eval_b0 + t, eval_out[t]);
+            if (eval_done.fetch_add(e - k, std::memory_order_acq_rel) + (e - k) == eval_len)
+              ready.store(r, std::memory_order_release);
+          }
+          acks.fetch_add(1, std::memory_order_acq_rel);
+        }
+      } else {  // the replay, in the exact order of Alg 3
+        request(0, nullptr);
+        for (int64_t b = 0; b < nblocks && nclusters > 0; ++b) {
+          wait_ready(b);
+          if (b > 0) {  // rotate: the previous block's keys / merges become "previous"
+            kset[kprev].clear();
+            std::swap(kprev, kcur);
+            std::memset(fbits[fprev], 0, sizeof(fbits[fprev]));
+            std::swap(fprev, fcur);
+          }
+          const bool overflow_prev = overflow;
+          overflow = false;
+          if (b + 1 < nblocks) request(b + 1, b > 0 ? &kset[kprev].keys() : nullptr);
+          const Pre* pr = ring[b & 1].data();
+          const size_t b0 = (size_t)b * BS, b1 = std::min(init_pos, b0 + BS);
+          for (size_t c = b0; c < b1 && nclusters > 0;) {
+            if (!extra.empty() && !before(init[c], extra.top())) {  // a re-inserted pair pops first
+              const int32_t i = (int32_t)extra.top().i, j = (int32_t)extra.top().j;
+              extra.pop();
+              process_pipe(i, j);
+              continue;
+            }
+            const Pre& p = pr[c - b0];
+            const int32_t i = (int32_t)init[c].i, j = (int32_t)init[c].j;
+            ++c;
+            if (p.cls == 1) {
+              ++n_spec_used;
+              continue;
+            }
+            if ((p.cls == 2 || p.cls == 3) && !fmod(p.ri) && !fmod(p.rj)) {
+              ++n_spec_used;
+              if (p.cls == 2) continue;
+              const uint32_t lo = (uint32_t)std::min(p.ri, p.rj), hi = (uint32_t)std::max(p.ri, p.rj);
+              const uint64_t key = ((uint64_t)lo << 32) | hi;
+              if (kset[kcur].contains(key) || kset[kprev].contains(key) ||
+                  ((overflow || overflow_prev) && members.contains(key)))
+                continue;  // re-inserted since this block's evaluation began
+              Cand cc;
+              cc.i = lo;
+              cc.j = hi;
+              cc.inter = p.inter;
+              cc.uni = p.uni;
+              reinsert_pipe(cc, key);
+              continue;
+            }
+            process_pipe(i, j);
+          }
+        }
+        // the cursor is done: the remaining re-inserted pairs with J > 0
+        while (!extra.empty() && nclusters > 0) {
+          const int32_t i = (int32_t)extra.top().i, j = (int32_t)extra.top().j;
+          extra.pop();
+          process_pipe(i, j);
+        }
+        stop.store(true, std::memory_order_release);
+      }
+    }
+    // hand the remaining key sets to the sequential structures of the J = 0 phase
+    for (int k = 0; k < 2; ++k) {
+      members.reserve_more(kset[k].keys().size());
+      for (uint64_t key : kset[k].keys()) members.insert(key);
+      kset[k].clear();
+    }
+    cur = init_pos;
+    blk0 = blk1 = init_pos;
+  }
   constexpr size_t PF = 32, PF2 = 16, PF3 = 8;  // prefetch distances (sequential mode)
   while (nclusters > 0) {
     int32_t i, j;
