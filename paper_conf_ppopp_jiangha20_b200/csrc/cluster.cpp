@@ -21,6 +21,7 @@
 // Readings R3-R12 decide everything the paper leaves open.
 #include <algorithm>
 #include <atomic>
+#include <thread>
 #include <chrono>
 #include <cstdio>
 #include <cstdlib>
@@ -513,7 +514,7 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
   // the sets of the previous and the current block only.
   int nthr = 1;
 #ifdef _OPENMP
-  nthr = omp_get_max_threads();
+  nthr = std::min(omp_get_max_threads(), 8);  // a few evaluators keep ahead of the replay
 #endif
   if (spec && nthr >= 3 && init_pos > 0 && getenv("SR_CLUSTER_NOPIPE") == nullptr) {
     const int64_t nblocks = (int64_t)((init_pos + BS - 1) / BS);
@@ -536,7 +537,15 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
     const uint64_t* flush_keys = nullptr;
     int64_t flush_n = 0, eval_b0 = 0, eval_len = 0;
     Pre* eval_out = nullptr;
-    auto pause = [] { __builtin_ia32_pause(); };
+    // spin briefly, then yield the core (the team may share cores with other threads)
+    auto pause = [] {
+      thread_local unsigned spins = 0;
+      if (++spins & 1023u)
+        __builtin_ia32_pause();
+      else
+        std::this_thread::yield();
+    };
+    std::atomic<int> team{0};
     auto cand_pipe = [&](uint64_t key) {
       return kset[kcur].contains(key) || kset[kprev].contains(key) || is_candidate_big(key);
     };
@@ -616,7 +625,7 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
     // publish the next evaluation (the evaluators are idle: the previous one has completed)
     auto request = [&](int64_t b, const std::vector<uint64_t>* keys) {
       if (b > 0)  // every evaluator has left the previous request's loops
-        while (acks.load(std::memory_order_acquire) < nthr - 1) pause();
+        while (acks.load(std::memory_order_acquire) < team.load(std::memory_order_relaxed) - 1) pause();
       acks.store(0, std::memory_order_relaxed);
       flush_n = keys ? (int64_t)keys->size() : 0;
       members.reserve_more((size_t)flush_n + (size_t)BS * 4 + 65536);
@@ -633,11 +642,17 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
     };
     auto wait_ready = [&](int64_t b) {
       const double te = dbg ? now() : 0.0;
+      if (team.load(std::memory_order_relaxed) < 2) {  // the runtime gave no evaluator thread
+        for (int64_t t = flush_cur.load(); t < flush_n; ++t) members.insert_distinct_concurrent(flush_keys[t]);
+        for (int64_t t = 0; t < eval_len; ++t) evaluate_one(eval_b0 + t, eval_out[t]);
+        ready.store(b, std::memory_order_release);
+      }
       while (ready.load(std::memory_order_acquire) != b) pause();
       if (dbg) t_eval += now() - te;  // time the replay waited for the evaluators
     };
 #pragma omp parallel num_threads(nthr)
     {
+      if (omp_get_thread_num() == 0) team.store(omp_get_num_threads(), std::memory_order_release);
       if (omp_get_thread_num() != 0) {  // evaluators
         int64_t seen = -1;
         while (true) {
