@@ -514,7 +514,7 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
   // the sets of the previous and the current block only.
   int nthr = 1;
 #ifdef _OPENMP
-  nthr = std::min(omp_get_max_threads(), 8);  // a few evaluators keep ahead of the replay
+  nthr = std::min(omp_get_max_threads(), 16);
 #endif
   if (spec && nthr >= 3 && init_pos > 0 && getenv("SR_CLUSTER_NOPIPE") == nullptr) {
     const int64_t nblocks = (int64_t)((init_pos + BS - 1) / BS);
@@ -530,21 +530,31 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
       return ((fbits[fprev][b >> 6] | fbits[fcur][b >> 6]) >> (b & 63)) & 1ull;
     };
     bool overflow = false;  // a block's key set was flushed early: re-check class 3 against `members`
+    // work cursors tagged with their request (request << 40 | position): a thread still looking
+    // at an earlier request can never claim work of a newer one, so no request waits for
+    // stragglers; a request is issued only after the previous one completed (all its claimed
+    // chunks counted)
+    constexpr int kTag = 40;
+    constexpr uint64_t kPos = (1ull << kTag) - 1;
     std::atomic<int64_t> req{-1}, ready{-1};
-    std::atomic<int64_t> flush_cur{0}, flush_done{0}, eval_cur{0}, eval_done{0};
+    std::atomic<uint64_t> flush_cur{0}, eval_cur{0};
+    std::atomic<int64_t> flush_done{0}, eval_done{0};
     std::atomic<bool> stop{false};
-    std::atomic<int> acks{0};  // evaluators done with the current request (all must be before the next)
+    auto claim = [&](std::atomic<uint64_t>& c, int64_t r, int64_t len, int64_t step, int64_t* k) {
+      uint64_t v = c.load(std::memory_order_acquire);
+      while (true) {
+        if ((int64_t)(v >> kTag) != r || (int64_t)(v & kPos) >= len) return false;
+        if (c.compare_exchange_weak(v, v + (uint64_t)step, std::memory_order_acq_rel, std::memory_order_acquire)) {
+          *k = (int64_t)(v & kPos);
+          return true;
+        }
+      }
+    };
     const uint64_t* flush_keys = nullptr;
     int64_t flush_n = 0, eval_b0 = 0, eval_len = 0;
     Pre* eval_out = nullptr;
-    // spin briefly, then yield the core (the team may share cores with other threads)
-    auto pause = [] {
-      thread_local unsigned spins = 0;
-      if (++spins & 1023u)
-        __builtin_ia32_pause();
-      else
-        std::this_thread::yield();
-    };
+    // spin (the phase lasts about a second; yielding measured slower, r02l)
+    auto pause = [] { __builtin_ia32_pause(); };
     std::atomic<int> team{0};
     auto cand_pipe = [&](uint64_t key) {
       return kset[kcur].contains(key) || kset[kprev].contains(key) || is_candidate_big(key);
@@ -624,9 +634,6 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
     };
     // publish the next evaluation (the evaluators are idle: the previous one has completed)
     auto request = [&](int64_t b, const std::vector<uint64_t>* keys) {
-      if (b > 0)  // every evaluator has left the previous request's loops
-        while (acks.load(std::memory_order_acquire) < team.load(std::memory_order_relaxed) - 1) pause();
-      acks.store(0, std::memory_order_relaxed);
       flush_n = keys ? (int64_t)keys->size() : 0;
       members.reserve_more((size_t)flush_n + (size_t)BS * 4 + 65536);
       members.set_size(members.size() + (size_t)flush_n);
@@ -634,16 +641,16 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
       eval_b0 = b * (int64_t)BS;
       eval_len = std::min<int64_t>((int64_t)init_pos, eval_b0 + (int64_t)BS) - eval_b0;
       eval_out = ring[b & 1].data();
-      flush_cur.store(0, std::memory_order_relaxed);
       flush_done.store(0, std::memory_order_relaxed);
-      eval_cur.store(0, std::memory_order_relaxed);
       eval_done.store(0, std::memory_order_relaxed);
+      flush_cur.store((uint64_t)b << kTag, std::memory_order_release);
+      eval_cur.store((uint64_t)b << kTag, std::memory_order_release);
       req.store(b, std::memory_order_release);
     };
     auto wait_ready = [&](int64_t b) {
       const double te = dbg ? now() : 0.0;
       if (team.load(std::memory_order_relaxed) < 2) {  // the runtime gave no evaluator thread
-        for (int64_t t = flush_cur.load(); t < flush_n; ++t) members.insert_distinct_concurrent(flush_keys[t]);
+        for (int64_t t = 0; t < flush_n; ++t) members.insert_distinct_concurrent(flush_keys[t]);
         for (int64_t t = 0; t < eval_len; ++t) evaluate_one(eval_b0 + t, eval_out[t]);
         ready.store(b, std::memory_order_release);
       }
@@ -660,23 +667,21 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
           while ((r = req.load(std::memory_order_acquire)) == seen && !stop.load(std::memory_order_acquire)) pause();
           if (r == seen) break;
           seen = r;
-          for (;;) {
-            const int64_t k = flush_cur.fetch_add(512, std::memory_order_relaxed);
-            if (k >= flush_n) break;
+          int64_t k;
+          while (claim(flush_cur, r, flush_n, 512, &k)) {
             const int64_t e = std::min(flush_n, k + 512);
             for (int64_t t = k; t < e; ++t) members.insert_distinct_concurrent(flush_keys[t]);
             flush_done.fetch_add(e - k, std::memory_order_release);
           }
-          while (flush_done.load(std::memory_order_acquire) < flush_n) pause();
-          for (;;) {
-            const int64_t k = eval_cur.fetch_add(64, std::memory_order_relaxed);
-            if (k >= eval_len) break;
+          // every flush chunk of this request is in before any of its evaluation reads `members`
+          while (req.load(std::memory_order_acquire) == r && flush_done.load(std::memory_order_acquire) < flush_n)
+            pause();
+          while (claim(eval_cur, r, eval_len, 64, &k)) {
             const int64_t e = std::min(eval_len, k + 64);
             for (int64_t t = k; t < e; ++t) evaluate_one(eval_b0 + t, eval_out[t]);
             if (eval_done.fetch_add(e - k, std::memory_order_acq_rel) + (e - k) == eval_len)
               ready.store(r, std::memory_order_release);
           }
-          acks.fetch_add(1, std::memory_order_acq_rel);
         }
       } else {  // the replay, in the exact order of Alg 3
         request(0, nullptr);

@@ -52,17 +52,6 @@ struct Frag<4> {
   __device__ __forceinline__ void store_cs(float* p) const { __stcs(reinterpret_cast<float4*>(p), v); }
 };
 template <>
-struct Frag<2> {
-  float2 v;
-  __device__ __forceinline__ void zero() { v = make_float2(0.f, 0.f); }
-  __device__ __forceinline__ void load_g(const float* p) { v = __ldg(reinterpret_cast<const float2*>(p)); }
-  __device__ __forceinline__ void load_cg(const float* p) { v = __ldcg(reinterpret_cast<const float2*>(p)); }
-  __device__ __forceinline__ void fma(float a, const Frag& b) { v.x = fmaf(a, b.v.x, v.x); v.y = fmaf(a, b.v.y, v.y); }
-  __device__ __forceinline__ void add(const Frag& b) { v.x += b.v.x; v.y += b.v.y; }
-  __device__ __forceinline__ void store(float* p) const { *reinterpret_cast<float2*>(p) = v; }
-  __device__ __forceinline__ void store_cs(float* p) const { __stcs(reinterpret_cast<float2*>(p), v); }
-};
-template <>
 struct Frag<1> {
   float v;
   __device__ __forceinline__ void zero() { v = 0.f; }
