@@ -1,15 +1,17 @@
 // sm_100a SpMM / SDDMM execution over an ASpT plan (Alg 1, Alg 2
 // P:78-92, row-wise GPU mapping P:101, adaptive sparse tiling P:111, Fig 5).
 //
-// Phase D ("dense tiles"): one CTA per row panel that has dense columns.  The B/Y
-//   rows of the panel's dense columns are staged into shared memory tile by tile with
-//   bulk asynchronous copies (cp.async.bulk -> UBLKCP, completion on an mbarrier with
-//   transaction counts), double-buffered so tile t+1 streams in while tile t is used.
-//   Warp w owns panel rows w, w+W, ...; each dense nnz is served from shared memory.
-// Phase S ("sparse remainder"): one warp per work item = a remainder row
-//   in round-2 order (perm2) or a bounded chunk of a long row; lanes own 16-byte column
-//   fragments, so every gathered B/Y row is one coalesced 128-bit load per lane; U gathers
-//   are in flight per lane.  SDDMM reduces each dot product with warp shuffles.
+// Phase D ("dense tiles"), two engines chosen by the plan's panel height:
+//   * panels of > 8 rows: persistent CTAs, a producer warp stages each tile's dense-column rows
+//     of B / Y into a shared-memory ring with TMA tile::gather4 (UTMALDG) and bulk copies
+//     completing on mbarriers; 8 consumer warps read them per nnz (spmm_dense_kernel,
+//     sddmm_dense_kernel);
+//   * panels of <= 8 rows: register tiles, one warp per panel keeps every row's accumulator in
+//     registers and gathers each dense column's row once (spmm_rtile_kernel, sddmm_rtile_kernel).
+// Phase S ("sparse remainder"): row-group tasks in perm2 order, one warp per task,
+//   gathers in flight across row boundaries; lanes own 16-byte column fragments, so every
+//   gathered row is one coalesced 128-bit load per lane (spmm_task_kernel, sddmm_task_kernel);
+//   one-row-per-warp kernels for other K (spmm_sparse_kernel, sddmm_sparse_kernel).
 // Lane geometry: LPG lanes cover LPG·VEC columns of one nnz; G = 32/LPG groups of a warp
 //   work on G different nnz at once (K = 32 -> 4 nnz per warp instruction).
 #include <cuda.h>  // CUtensorMap
