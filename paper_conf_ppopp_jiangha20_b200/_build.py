@@ -36,7 +36,9 @@ def _compile(src: str, verbose: bool) -> str:
     if not _stale(o, s):
         return o
     if src.endswith(".cu"):
-        cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xptxas", "-v" if verbose else "-O3",
+        # SR_NVCC_DEFS: extra -D flags for measurement builds (compile-time knobs in exec.cu)
+        defs = os.environ.get("SR_NVCC_DEFS", "").split()
+        cmd = [NVCC, *ARCH, *defs, "-O3", "-lineinfo", "-std=c++17", "-Xptxas", "-v" if verbose else "-O3",
                "-Xcompiler", "-fPIC,-fopenmp,-O3", "-I", os.path.join(ROOT, "include"), "-c", s, "-o", o]
     else:
         cmd = ["g++", "-O3", "-std=c++17", "-fPIC", "-fopenmp", "-I", os.path.join(CUDA, "include"),

@@ -185,6 +185,8 @@ int upload_items(DevPlan& P, ItemBuilder& ib, int64_t n_sddmm_items, cudaStream_
   const std::vector<int4> stasks = build_tasks(ib, n_sddmm_items, 8);
   P.n_stasks = (int64_t)stasks.size();
   SR_TRY(P.stasks.upload(stasks, s));
+  SR_TRY(P.task_ticket.alloc(2));
+  SR_CUDA_TRY(cudaMemsetAsync(P.task_ticket.p, 0, 2 * sizeof(int32_t), s));
   P.n_items = (int64_t)ib.items.size();
   P.n_sitems = n_sddmm_items;
   SR_TRY(P.items.upload(ib.items, s));

@@ -323,17 +323,15 @@ __device__ __forceinline__ void task_store(Frag<VEC> v, uint32_t o, float* __res
 
 // VEC 4: a launch covers 128 columns (one float4 per lane); VEC 1: 32 columns (K = 32·passes,
 // one float per lane, 128-byte gathers).  The host offsets B and C per pass; ldb is in bytes.
-template <int U, int MINB, int VEC>
-__global__ void __launch_bounds__(256, MINB) spmm_task_kernel(
-    const int4* __restrict__ tasks, int64_t n_tasks, const Item* __restrict__ items,
+template <int U, int VEC>
+__device__ __forceinline__ void spmm_task(
+    int64_t w, const int4* __restrict__ tasks, const Item* __restrict__ items,
     const uint32_t* __restrict__ meta, const int2* __restrict__ ent, const float* __restrict__ B, uint32_t ldb,
     float* __restrict__ C, int64_t ldc, int K, int k0, float* __restrict__ scratch,
     const int2* __restrict__ split_info, int* __restrict__ split_counter) {
   const int lane = threadIdx.x & 31;
   // warp-uniform values through lane-0 shuffles, so the compiler sees uniform control flow
   // (no divergent-shuffle fallback paths and no stack frame)
-  const int64_t w = (int64_t)blockIdx.x * (blockDim.x >> 5) + __shfl_sync(FULL, threadIdx.x >> 5, 0);
-  if (w >= n_tasks) return;
   int4 t = __ldg(tasks + w);  // {e0, e1, first item, end item}
   t.x = __shfl_sync(FULL, t.x, 0); t.y = __shfl_sync(FULL, t.y, 0);
   t.z = __shfl_sync(FULL, t.z, 0); t.w = __shfl_sync(FULL, t.w, 0);
@@ -422,6 +420,48 @@ __global__ void __launch_bounds__(256, MINB) spmm_task_kernel(
   }
 }
 
+// Work distribution of the task kernels: each warp draws task indices from a ticket counter in
+// task (perm2) order until they run out, so a warp that finishes early takes the next task
+// instead of idling until its CTA's slowest warp is done (one task per warp left C2 SDDMM at
+// 37 % warps active of a 50 % occupancy limit, profiles/r02).  The next ticket is drawn while
+// the current task runs.  Every warp draws exactly one ticket past the last task; the warp
+// holding the final ticket (n_tasks + warps - 1) resets the counter for the next launch.
+__device__ __forceinline__ int64_t first_ticket(int* ticket) {
+  int v = 0;
+  if ((threadIdx.x & 31) == 0) v = atomicAdd(ticket, 1);
+  return __shfl_sync(FULL, v, 0);
+}
+__device__ __forceinline__ int draw_ticket(int* ticket) {
+  return (threadIdx.x & 31) == 0 ? atomicAdd(ticket, 1) : 0;
+}
+__device__ __forceinline__ void last_ticket_reset(int* ticket, int64_t w, int64_t n_tasks) {
+  const int64_t nw = (int64_t)gridDim.x * (blockDim.x >> 5);
+  if ((threadIdx.x & 31) == 0 && w == n_tasks + nw - 1) *ticket = 0;
+}
+
+// DYN false: one task per warp in launch order (task b·8 + w on warp w of CTA b: consecutive,
+// similar rows share an SM and its L1), the measured-faster choice for the SpMM kernels and K = 32.
+template <int U, int MINB, int VEC, bool DYN>
+__global__ void __launch_bounds__(256, MINB) spmm_task_kernel(
+    const int4* __restrict__ tasks, int64_t n_tasks, const Item* __restrict__ items,
+    const uint32_t* __restrict__ meta, const int2* __restrict__ ent, const float* __restrict__ B, uint32_t ldb,
+    float* __restrict__ C, int64_t ldc, int K, int k0, float* __restrict__ scratch,
+    const int2* __restrict__ split_info, int* __restrict__ split_counter, int* __restrict__ ticket) {
+  if constexpr (!DYN) {
+    const int64_t w = (int64_t)blockIdx.x * (blockDim.x >> 5) + __shfl_sync(FULL, threadIdx.x >> 5, 0);
+    if (w < n_tasks)
+      spmm_task<U, VEC>(w, tasks, items, meta, ent, B, ldb, C, ldc, K, k0, scratch, split_info, split_counter);
+    return;
+  }
+  int64_t w = first_ticket(ticket);
+  while (w < n_tasks) {
+    const int nxt = draw_ticket(ticket);
+    spmm_task<U, VEC>(w, tasks, items, meta, ent, B, ldb, C, ldc, K, k0, scratch, split_info, split_counter);
+    w = __shfl_sync(FULL, nxt, 0);
+  }
+  last_ticket_reset(ticket, w, n_tasks);
+}
+
 // ------------------------------------------------------------------ phase S: SDDMM, row-group tasks
 // One warp per task = up to kSddmmTaskRows consecutive remainder rows (or one chunk of a long
 // row) with at most task_nnz entries.  At task start the lanes copy the task's X rows into the
@@ -438,17 +478,13 @@ __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wai
 
 // PERM: lane 8g+k holds batch entry 4k+g, so in step s group g's entry (4s+g) sits in its own
 // lane 8g+s, which stores the result from its own registers (no value / index shuffles).
-template <int NCH, int U, int MINB, bool PERM = false>
-__global__ void __launch_bounds__(256, MINB) sddmm_task_kernel(
-    const int4* __restrict__ tasks, int64_t n_tasks, const Item* __restrict__ items, const int2* __restrict__ ent,
-    const int32_t* __restrict__ oidx, const float* __restrict__ X, int64_t ldx, const float* __restrict__ Y,
-    uint32_t ldy_bytes, float* __restrict__ out) {
+template <int NCH, int U, bool PERM>
+__device__ __forceinline__ void sddmm_task(
+    int64_t w, float4 (*xs)[NCH * 8], const int4* __restrict__ tasks, const Item* __restrict__ items,
+    const int2* __restrict__ ent, const int32_t* __restrict__ oidx, const float* __restrict__ X, int64_t ldx,
+    const float* __restrict__ Y, uint32_t ldy_bytes, float* __restrict__ out) {
   constexpr int G = 4, LPG = 8;
-  __shared__ float4 xs[8][kSddmmTaskRows][NCH * 8];
   const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
-  const int wid = __shfl_sync(FULL, threadIdx.x >> 5, 0);
-  const int64_t w = (int64_t)blockIdx.x * (blockDim.x >> 5) + wid;
-  if (w >= n_tasks) return;
   int4 t = __ldg(tasks + w);  // {e0, e1, first item, end item}; warp-uniform via lane-0 shuffles
   t.x = __shfl_sync(FULL, t.x, 0); t.y = __shfl_sync(FULL, t.y, 0);
   t.z = __shfl_sync(FULL, t.z, 0); t.w = __shfl_sync(FULL, t.w, 0);
@@ -466,7 +502,7 @@ __global__ void __launch_bounds__(256, MINB) sddmm_task_kernel(
   }
   for (int r = 0; r < cnt; ++r) {  // stage the task's X rows (K·4 bytes each) in shared memory
     const int xr = __shfl_sync(FULL, xrow, r);
-    if (lane < NCH * 8) cp_async_cg16(&xs[wid][r][lane], X + (int64_t)xr * ldx + lane * 4);
+    if (lane < NCH * 8) cp_async_cg16(&xs[r][lane], X + (int64_t)xr * ldx + lane * 4);
   }
   asm volatile("cp.async.commit_group;" ::: "memory");
   const char* Yl = reinterpret_cast<const char*>(Y + lg * 4);
@@ -506,7 +542,7 @@ __global__ void __launch_bounds__(256, MINB) sddmm_task_kernel(
         if (row[u] != cur) {
           cur = row[u];
 #pragma unroll
-          for (int ch = 0; ch < NCH; ++ch) x[ch] = xs[wid][cur][ch * 8 + lg];
+          for (int ch = 0; ch < NCH; ++ch) x[ch] = xs[cur][ch * 8 + lg];
         }
         float d = 0.f;
 #pragma unroll
@@ -532,6 +568,28 @@ __global__ void __launch_bounds__(256, MINB) sddmm_task_kernel(
       }
     }
   }
+}
+
+template <int NCH, int U, int MINB, bool PERM, bool DYN>
+__global__ void __launch_bounds__(256, MINB) sddmm_task_kernel(
+    const int4* __restrict__ tasks, int64_t n_tasks, const Item* __restrict__ items, const int2* __restrict__ ent,
+    const int32_t* __restrict__ oidx, const float* __restrict__ X, int64_t ldx, const float* __restrict__ Y,
+    uint32_t ldy_bytes, float* __restrict__ out, int* __restrict__ ticket) {
+  __shared__ float4 xs[8][kSddmmTaskRows][NCH * 8];
+  const int wid = __shfl_sync(FULL, threadIdx.x >> 5, 0);
+  if constexpr (!DYN) {
+    const int64_t w = (int64_t)blockIdx.x * (blockDim.x >> 5) + wid;
+    if (w < n_tasks) sddmm_task<NCH, U, PERM>(w, xs[wid], tasks, items, ent, oidx, X, ldx, Y, ldy_bytes, out);
+    return;
+  }
+  int64_t w = first_ticket(ticket);
+  while (w < n_tasks) {
+    const int nxt = draw_ticket(ticket);
+    sddmm_task<NCH, U, PERM>(w, xs[wid], tasks, items, ent, oidx, X, ldx, Y, ldy_bytes, out);
+    w = __shfl_sync(FULL, nxt, 0);
+    __syncwarp();  // every lane's reads of the staged X rows precede the next task's staging
+  }
+  last_ticket_reset(ticket, w, n_tasks);
 }
 
 // ------------------------------------------------------------------ phase D: register tiles
@@ -744,11 +802,22 @@ __global__ void __launch_bounds__(256) sddmm_rtile_scalar_kernel(
 // an empty mbarrier, so consumers never meet at a CTA barrier and unit boundaries cost no
 // pipeline drain: unit n+1's tiles stream in while unit n's results are stored.
 // Consumer warp w owns the contiguous panel rows [w·RPW, (w+1)·RPW).
-constexpr int kDenseWarps = 8;  // consumer warps per phase-D CTA (+1 producer warp)
-constexpr int kMaxStages = 3;   // SpMM runs 3 stages, SDDMM 2 (its stages also carry output indices)
-constexpr int kSpmmStages = 3;
-constexpr int kSddmmStages = 2;
-constexpr int kDenseCtasPerSM = 2;
+// (SR_DENSE_WARPS / SR_SPMM_STAGES / SR_DENSE_CTAS: compile-time measurement knobs, see
+// profiles/r02/NOTES.md; the defaults are the measured choice)
+#ifndef SR_DENSE_WARPS
+#define SR_DENSE_WARPS 8
+#endif
+#ifndef SR_SPMM_STAGES
+#define SR_SPMM_STAGES 3
+#endif
+#ifndef SR_DENSE_CTAS
+#define SR_DENSE_CTAS 2
+#endif
+constexpr int kDenseWarps = SR_DENSE_WARPS;  // consumer warps per phase-D CTA (+1 producer warp)
+constexpr int kSpmmStages = SR_SPMM_STAGES;
+constexpr int kSddmmStages = 2;               // SDDMM stages also carry output indices
+constexpr int kMaxStages = kSpmmStages > kSddmmStages ? kSpmmStages : kSddmmStages;
+constexpr int kDenseCtasPerSM = SR_DENSE_CTAS;
 constexpr size_t kUnitBlobBytes = kMaxUnitBlobBytes;  // DUnit + VTiles + dense column ids
 
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
@@ -1249,6 +1318,36 @@ int num_sms() {
   return n;
 }
 
+// Grid of a ticket-driven task kernel: the CTAs the device holds at once (occupancy × SMs, cached
+// per kernel and device), or fewer when there are fewer tasks.
+unsigned resident_grid(const void* kern, int64_t n_tasks) {
+  static std::mutex mu;
+  static std::map<std::pair<const void*, int>, int> occ;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  int per_sm = 0;
+  {
+    std::lock_guard<std::mutex> lock(mu);
+    auto it = occ.find({kern, dev});
+    if (it == occ.end()) {
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kSparseWarps * 32, 0) != cudaSuccess ||
+          per_sm < 1)
+        per_sm = 1;
+      occ[{kern, dev}] = per_sm;
+    } else {
+      per_sm = it->second;
+    }
+  }
+  const int64_t need = (n_tasks + kSparseWarps - 1) / kSparseWarps;
+  return (unsigned)std::max<int64_t>(1, std::min<int64_t>(need, (int64_t)per_sm * num_sms()));
+}
+
+int dense_rows_per_warp(int panel_rows) {
+  int r = 2;
+  while (r < 16 && r * kDenseWarps < panel_rows) r <<= 1;
+  return r;
+}
+
 template <int LPG, int VEC>
 int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int64_t ldc,
              cudaStream_t s, int32_t* launches) {
@@ -1300,11 +1399,12 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
       return SR_OK;
     };
     if (P.profiling) SR_TRY(prof_begin(P, 1, s));
-    if (P.panel_rows <= 8 * kDenseWarps) {
-      SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 8>));
-    } else {
-      SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 16>));
-    }
+    // rows per consumer warp: the smallest of 2, 4, 8, 16 that covers the panel
+    const int rpw = dense_rows_per_warp(P.panel_rows);
+    if (rpw <= 2) SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 2>));
+    else if (rpw <= 4) SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 4>));
+    else if (rpw <= 8) SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 8>));
+    else SR_TRY(launch(spmm_dense_kernel<LPG, VEC, UD, 16>));
     if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;
   }
@@ -1318,18 +1418,18 @@ int run_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int6
     // row-group task kernels: K = 128·passes (float4 lanes) or 32·passes (float lanes)
     const int tvec = (VEC == 4 && K % 128 == 0) ? 4 : (K % 32 == 0 ? 1 : 0);
     if (tvec && ldb * 4 < (1ll << 32) && task_kernels() && P.n_tasks > 0) {
-      const unsigned tgrid = (unsigned)((P.n_tasks + kSparseWarps - 1) / kSparseWarps);
       const int pass = 32 * tvec;
       auto tk = [&](auto kern) {
+        const unsigned tgrid = (unsigned)((P.n_tasks + kSparseWarps - 1) / kSparseWarps);
         for (int k0 = 0; k0 < K; k0 += pass)
           kern<<<tgrid, kSparseWarps * 32, 0, s>>>(P.tasks.p, P.n_tasks, P.items.p, P.item_meta.p, P.s_ent.p,
                                                     B + k0, (uint32_t)(ldb * 4), C + k0, ldc, (int)K, k0, P.scratch.p,
-                                                    P.split_info.p, P.split_counter.p);
+                                                    P.split_info.p, P.split_counter.p, P.task_ticket.p);
       };
       if (tvec == 4)
-        tk(spmm_task_kernel<4, 8, 4>);  // U 4 gathers per lane, 8 CTAs (64 warps) per SM
+        tk(spmm_task_kernel<4, 8, 4, false>);  // U 4 gathers per lane, 8 CTAs (64 warps) per SM
       else
-        tk(spmm_task_kernel<8, 8, 1>);
+        tk(spmm_task_kernel<8, 8, 1, false>);
       SR_CUDA_TRY(cudaGetLastError());
       if (P.profiling) SR_TRY(prof_end(P, s));
       ++*launches;
@@ -1389,7 +1489,10 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
     };
     constexpr int UD = 4;
     if (P.profiling) SR_TRY(prof_begin(P, 3, s));
-    if (P.panel_rows <= 8 * kDenseWarps) SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 8>));
+    const int rpw = dense_rows_per_warp(P.panel_rows);
+    if (rpw <= 2) SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 2>));
+    else if (rpw <= 4) SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 4>));
+    else if (rpw <= 8) SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 8>));
     else SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 16>));
     if (P.profiling) SR_TRY(prof_end(P, s));
     ++*launches;
@@ -1399,13 +1502,17 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
     if (P.profiling) SR_TRY(prof_begin(P, 4, s));
     if (LPG == 8 && VEC == 4 && NCH <= 4 && K == 32 * NCH && ldy * 4 < (1ll << 32) && task_kernels() &&
         P.n_stasks > 0) {
-      const unsigned tgrid = (unsigned)((P.n_stasks + kSparseWarps - 1) / kSparseWarps);
-      auto tk = [&](auto kern) {
+      auto tk = [&](auto kern, bool dyn) {
+        const unsigned tgrid = dyn ? resident_grid(reinterpret_cast<const void*>(kern), P.n_stasks)
+                                   : (unsigned)((P.n_stasks + kSparseWarps - 1) / kSparseWarps);
         kern<<<tgrid, kSparseWarps * 32, 0, s>>>(P.stasks.p, P.n_stasks, P.items.p, P.s_ent.p, P.s_oidx.p, X,
-                                                  ldx, Y, (uint32_t)(ldy * 4), out);
+                                                  ldx, Y, (uint32_t)(ldy * 4), out, P.task_ticket.p + 1);
       };
       constexpr int NC = NCH > 4 ? 4 : NCH;  // (NCH <= 4 guarded above; keeps NCH 8 instantiable)
-      tk(sddmm_task_kernel<NC, 2, 4, true>);
+      // K = 128: ticket-driven warps (C2: 0.637 -> 0.547 ms under ncu, warps active 37 -> 49 %);
+      // K = 32 measured slower that way (0.283 -> 0.325 ms), K = 64 unmeasured: launch order
+      if constexpr (NC == 4) tk(sddmm_task_kernel<NC, 2, 4, true, true>, true);
+      else tk(sddmm_task_kernel<NC, 2, 4, true, false>, false);
       SR_CUDA_TRY(cudaGetLastError());
       if (P.profiling) SR_TRY(prof_end(P, s));
       ++*launches;

@@ -212,6 +212,7 @@ struct DevPlan {
   DevBuf<int4> tasks;         // SpMM row-group tasks {e0, e1, first item, end item} (build_tasks)
   int64_t n_tasks = 0;
   DevBuf<int4> stasks;        // SDDMM row-group tasks (<= 8 rows each, non-empty rows only)
+  DevBuf<int32_t> task_ticket;  // [0] SpMM, [1] SDDMM task kernels' work counters (exec.cu: first_ticket)
   int64_t n_stasks = 0;
   DevBuf<Item> sitems;        // SDDMM items (remainder rows / chunks only)
   int64_t n_sitems = 0;

@@ -223,6 +223,26 @@ def test_unsorted_input_keeps_caller_nnz_order(env, oracle):
             np.testing.assert_array_equal(U.colidx[t["r_pos"]], t["r_col"])
 
 
+@pytest.mark.parametrize("K", [32, 128])
+def test_repeated_launches_fresh_results(env, oracle, K):
+    """Consecutive SpMM / SDDMM calls on one handle, each with new operands into a poisoned
+    output: every call must compute every task (the K = 128 SDDMM kernel hands tasks out through a
+    ticket counter that its last warp resets for the next launch, exec.cu: first_ticket)."""
+    sr, torch = env
+    A = g.rmat(scale=17)  # 2.1 M nnz: ~10^4 tasks, several per warp of the resident grid
+    M = sr.SparseMatrix.from_csr(A)
+    for it in range(3):
+        B = g.dense(A.ncols, K, seed=20 + it)
+        X, Y = g.dense(A.nrows, K, seed=20 + it, stream=1), g.dense(A.ncols, K, seed=20 + it, stream=2)
+        C = torch.full((A.nrows, K), float("nan"), device="cuda")
+        out = torch.full((A.nnz,), float("nan"), device="cuda")
+        M.spmm(torch.from_numpy(B).cuda(), C)
+        M.sddmm(torch.from_numpy(X).cuda(), torch.from_numpy(Y).cuda(), out)
+        torch.cuda.synchronize()
+        _spmm_check(oracle, A, B, C.cpu().numpy())
+        _sddmm_check(oracle, A, X, Y, out.cpu().numpy())
+
+
 def test_strided_and_misaligned_operands(env, oracle):
     sr, torch = env
     A = g.random_csr(150, 100, 0.08, 4, empty_frac=0.1)
