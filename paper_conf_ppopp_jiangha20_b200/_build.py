@@ -53,9 +53,16 @@ def _compile(src: str, verbose: bool) -> str:
 
 
 def build(verbose: bool = False, force: bool = False) -> str:
+    # objects built with other SR_NVCC_DEFS (a measurement build) are never reused
+    stamp = os.path.join(BUILD, "nvcc_defs.txt")
+    defs = os.environ.get("SR_NVCC_DEFS", "")
+    if os.path.isdir(BUILD) and (not os.path.exists(stamp) or open(stamp).read() != defs):
+        force = True
     if force and os.path.isdir(BUILD):
         shutil.rmtree(BUILD)
     os.makedirs(BUILD, exist_ok=True)
+    with open(stamp, "w") as f:
+        f.write(defs)
     with cf.ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 2)) as ex:
         objs = list(ex.map(lambda s: _compile(s, verbose), CU + CPP))
     if os.path.exists(OUT) and all(os.path.getmtime(OUT) >= os.path.getmtime(o) for o in objs):

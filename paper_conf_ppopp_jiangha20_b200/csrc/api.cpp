@@ -862,8 +862,13 @@ int sr_reorder(sr_csr h, const sr_reorder_params* p, sr_stream stream) {
   double t0 = now_s();
   const int32_t dense_min0 = p->auto_dense_min > 0 ? p->auto_dense_min : p->dense_min;
   Tiling t_id;
-  tile_rows(A, ident, p->panel_rows, dense_min0, t_id);
-  st.dense0 = t_id.n_dense();
+  const bool tile_ident = p->mode == SR_REORDER_OFF;  // OFF plans are the identity tiling itself
+  if (tile_ident) {
+    tile_rows(A, ident, p->panel_rows, dense_min0, t_id);
+    st.dense0 = t_id.n_dense();
+  } else {  // only the count decides round 1 (the tiles are built below if it is skipped)
+    st.dense0 = dense_count(A, ident, p->panel_rows, dense_min0);
+  }
   st.t_tile_s += now_s() - t0;
   bool round1 = p->mode == SR_REORDER_FORCE;
   if (p->mode == SR_REORDER_AUTO)
@@ -877,7 +882,7 @@ int sr_reorder(sr_csr h, const sr_reorder_params* p, sr_stream stream) {
     st.t_tile_s += now_s() - t0;
   } else {
     h->perm1 = ident;
-    if (dense_min0 != p->dense_min) {  // the plan tiles with the execution threshold
+    if (!tile_ident || dense_min0 != p->dense_min) {  // the plan tiles with the execution threshold
       t0 = now_s();
       tile_rows(A, ident, p->panel_rows, p->dense_min, t_id);
       st.t_tile_s += now_s() - t0;

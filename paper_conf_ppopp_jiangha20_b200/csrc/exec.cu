@@ -798,14 +798,17 @@ __global__ void __launch_bounds__(256) sddmm_rtile_scalar_kernel(
 // unit of its CTA through an NST-deep shared-memory ring: the tile's B/Y rows (one
 // cp.async.bulk per dense column, 16-byte aligned, K·4 bytes), its panel-row offsets (trp),
 // its entry block (and SDDMM output indices) and a 32-byte stage header, all completing on
-// one full mbarrier with a transaction count.  Consumer warps (8) release stages through
+// one full mbarrier with a transaction count.  Consumer warps (16) release stages through
 // an empty mbarrier, so consumers never meet at a CTA barrier and unit boundaries cost no
 // pipeline drain: unit n+1's tiles stream in while unit n's results are stored.
-// Consumer warp w owns the contiguous panel rows [w·RPW, (w+1)·RPW).
+// Consumer warp w owns the contiguous panel rows [w·RPW, (w+1)·RPW), RPW the smallest of 2, 4, 8,
+// 16 that covers the panel (before r02t every panel ran RPW 8 or 16, so 16- and 32-row panels left
+// most consumer warps idle).  16 consumer warps (56 registers) measured faster than 8 (96):
+// C4 64-row panels, dense_min 8: 3.92 -> 3.56 ms per SpMM (r02t); 3 CTAs x 2 stages was slower.
 // (SR_DENSE_WARPS / SR_SPMM_STAGES / SR_DENSE_CTAS: compile-time measurement knobs, see
 // profiles/r02/NOTES.md; the defaults are the measured choice)
 #ifndef SR_DENSE_WARPS
-#define SR_DENSE_WARPS 8
+#define SR_DENSE_WARPS 16
 #endif
 #ifndef SR_SPMM_STAGES
 #define SR_SPMM_STAGES 3
@@ -823,7 +826,7 @@ constexpr size_t kUnitBlobBytes = kMaxUnitBlobBytes;  // DUnit + VTiles + dense 
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
-__device__ __forceinline__ void consumers_sync() {  // named barrier over the 8 consumer warps
+__device__ __forceinline__ void consumers_sync() {  // named barrier over the consumer warps
   asm volatile("bar.sync 1, %0;" ::"n"(kDenseWarps * 32) : "memory");
 }
 
@@ -1079,7 +1082,7 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) spmm_
       if (threadIdx.x == 0) last_ticket = (atomicAdd(split_counter + si.x, 1) == si.y - 1);
       consumers_sync();
       if (last_ticket) {
-        // all 256 consumer threads share the (row, fragment) sums; chunk partials are added
+        // all consumer threads share the (row, fragment) sums; chunk partials are added
         // in chunk order with 4 loads in flight (a hub panel can have >100 chunks)
         __threadfence();
         const int kq = (K + VEC - 1) / VEC;

@@ -259,6 +259,7 @@ namespace sr {
 void tile_rows(const HostCSR& A, const std::vector<int32_t>& perm, int32_t panel_rows,
                int32_t dense_min, Tiling& t);
 void avgsim_positions(const Tiling& t, uint64_t* num, uint64_t* den);
+int64_t dense_count(const HostCSR& A, const std::vector<int32_t>& perm, int32_t panel_rows, int32_t dense_min);
 // cluster.cpp
 void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t npairs,
                   const uint64_t* pairs, const uint32_t* inter, const uint32_t* uni,

@@ -123,6 +123,36 @@ void tile_rows(const HostCSR& A, const std::vector<int32_t>& perm, int32_t P, in
   }
 }
 
+// Dense nnz of the tiling of `perm` (= Tiling::n_dense() of tile_rows with the same arguments)
+// without building the tiles: the AUTO round-1 decision needs only this count.
+int64_t dense_count(const HostCSR& A, const std::vector<int32_t>& perm, int32_t P, int32_t dense_min) {
+  const int64_t M = A.M, N = A.N;
+  const int64_t npanels = (M + P - 1) / P;
+  int64_t total = 0;
+#pragma omp parallel reduction(+ : total)
+  {
+    std::vector<int32_t> cnt((size_t)N, 0);
+    std::vector<int32_t> touched;
+#pragma omp for schedule(dynamic, 16)
+    for (int64_t p = 0; p < npanels; ++p) {
+      const int64_t q0 = p * P, q1 = std::min<int64_t>(M, q0 + P);
+      touched.clear();
+      for (int64_t q = q0; q < q1; ++q) {
+        const int64_t r = perm[q];
+        for (int64_t e = A.rowptr[r]; e < A.rowptr[r + 1]; ++e) {
+          const int32_t c = A.col[e];
+          if (cnt[c]++ == 0) touched.push_back(c);
+        }
+      }
+      for (int32_t c : touched) {
+        if (cnt[c] >= dense_min) total += cnt[c];
+        cnt[c] = 0;
+      }
+    }
+  }
+  return total;
+}
+
 // AvgSim over the non-empty remainder rows in position order, each term
 // floor(2^32·inter/uni) (reading R27), exact integer sum.
 void avgsim_positions(const Tiling& t, uint64_t* num, uint64_t* den) {
