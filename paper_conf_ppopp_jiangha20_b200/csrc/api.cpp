@@ -656,8 +656,8 @@ int check_params(const sr_reorder_params* p) {
 // LSH + Alg 3 over a column-sorted CSR (rows = the matrix being reordered).
 int reorder_round(const int64_t* rowptr, const int32_t* col, int64_t M, const sr_reorder_params& p,
                   cudaStream_t s, std::vector<int32_t>& perm, int64_t* E, double* t_lsh, double* t_cl) {
-  std::vector<uint64_t> pairs, by_key;
-  std::vector<uint32_t> inter, uni;
+  HostVec<uint64_t> pairs, by_key;
+  HostVec<uint32_t> inter, uni;
   const double t0 = now_s();
   SR_TRY(lsh_candidates(rowptr, col, M, rowptr[M], p, s, pairs, inter, uni, E, &by_key));
   const double t1 = now_s();

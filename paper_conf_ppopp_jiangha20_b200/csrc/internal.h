@@ -5,6 +5,8 @@
 
 #include <cstdint>
 #include <string>
+#include <memory>
+#include <utility>
 #include <vector>
 
 #include "../../include/sr.h"
@@ -265,12 +267,36 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
                   const uint64_t* pairs, const uint32_t* inter, const uint32_t* uni,
                   int32_t threshold_size, int32_t* perm, const uint64_t* pairs_by_key = nullptr);
 void partition_panels(int64_t npanels, const int64_t* w, int32_t G, int64_t* cuts);
+// Host vector whose resize() leaves new elements uninitialised (a D2H copy overwrites them).
+template <class T>
+struct DefaultInitAlloc : std::allocator<T> {
+  template <class U>
+  struct rebind {
+    using other = DefaultInitAlloc<U>;
+  };
+  DefaultInitAlloc() = default;
+  template <class U>
+  DefaultInitAlloc(const DefaultInitAlloc<U>&) noexcept {}
+  template <class U>
+  void construct(U* p) noexcept {
+    ::new (static_cast<void*>(p)) U;
+  }
+  template <class U, class... A>
+  void construct(U* p, A&&... a) {
+    ::new (static_cast<void*>(p)) U(std::forward<A>(a)...);
+  }
+};
+template <class T>
+using HostVec = std::vector<T, DefaultInitAlloc<T>>;
+// Device -> pageable host copy through a pinned two-chunk staging ring, the chunk copies out of
+// the ring done by all host threads (first touch of the destination pages included); synchronous.
+int d2h_staged(void* dst, const void* src, size_t bytes, cudaStream_t s);
 // lsh.cu : device LSH candidate generation + exact Jaccard (sorted J order).
 // Returns candidate pairs sorted by (J desc, pair asc) with their (inter, uni).
 int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int64_t nnz,
-                   const sr_reorder_params& p, cudaStream_t s, std::vector<uint64_t>& pairs_by_j,
-                   std::vector<uint32_t>& inter, std::vector<uint32_t>& uni, int64_t* E,
-                   std::vector<uint64_t>* pairs_by_key = nullptr);
+                   const sr_reorder_params& p, cudaStream_t s, HostVec<uint64_t>& pairs_by_j,
+                   HostVec<uint32_t>& inter, HostVec<uint32_t>& uni, int64_t* E,
+                   HostVec<uint64_t>* pairs_by_key = nullptr);
 // exec.cu : launchers
 int launch_spmm(sr_csr_s* h, const float* B, int64_t K, int64_t ldb, float* C, int64_t ldc,
                 cudaStream_t s, int32_t* launches);

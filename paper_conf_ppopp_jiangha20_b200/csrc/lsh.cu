@@ -18,6 +18,8 @@
 #include <chrono>
 #include <cstdio>
 #include <cstdlib>
+#include <cstring>
+#include <mutex>
 #include <vector>
 
 #include "internal.h"
@@ -267,10 +269,49 @@ inline unsigned blocks(int64_t n, int t) { return (unsigned)std::max<int64_t>(1,
 
 }  // namespace
 
+int d2h_staged(void* dst, const void* src, size_t bytes, cudaStream_t s) {
+  // a pageable cudaMemcpy runs at a few GB/s through the driver's staging buffer and first-touches
+  // the destination on one thread (r02: 0.15 s for C2's 387 MB of candidates); here the PCIe copy
+  // of chunk i+1 overlaps the all-thread copy of chunk i out of a pinned ring
+  constexpr size_t kChunk = size_t(16) << 20;
+  static std::mutex mu;
+  static char* ring = nullptr;
+  static cudaEvent_t done[2];
+  std::lock_guard<std::mutex> lock(mu);
+  if (ring == nullptr) {
+    SR_CUDA_TRY(cudaMallocHost(reinterpret_cast<void**>(&ring), 2 * kChunk));
+    for (auto& e : done) SR_CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  }
+  const size_t n = (bytes + kChunk - 1) / kChunk;
+  auto issue = [&](size_t i) -> int {
+    const size_t off = i * kChunk, len = std::min(kChunk, bytes - off);
+    SR_CUDA_TRY(cudaMemcpyAsync(ring + (i & 1) * kChunk, static_cast<const char*>(src) + off, len,
+                                cudaMemcpyDeviceToHost, s));
+    SR_CUDA_TRY(cudaEventRecord(done[i & 1], s));
+    return SR_OK;
+  };
+  if (n > 0) SR_TRY(issue(0));
+  for (size_t i = 0; i < n; ++i) {
+    SR_CUDA_TRY(cudaEventSynchronize(done[i & 1]));
+    if (i + 1 < n) SR_TRY(issue(i + 1));  // its slot's previous chunk (i-1) was copied out below
+    const size_t off = i * kChunk, len = std::min(kChunk, bytes - off);
+    const char* from = ring + (i & 1) * kChunk;
+    char* to = static_cast<char*>(dst) + off;
+    constexpr size_t kPiece = size_t(1) << 20;
+    const int64_t np = (int64_t)((len + kPiece - 1) / kPiece);
+#pragma omp parallel for schedule(static)
+    for (int64_t k = 0; k < np; ++k) {
+      const size_t o = (size_t)k * kPiece;
+      std::memcpy(to + o, from + o, std::min(kPiece, len - o));
+    }
+  }
+  return SR_OK;
+}
+
 int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int64_t nnz,
-                   const sr_reorder_params& p, cudaStream_t s, std::vector<uint64_t>& pairs_by_j,
-                   std::vector<uint32_t>& inter_h, std::vector<uint32_t>& uni_h, int64_t* E_out,
-                   std::vector<uint64_t>* pairs_by_key) {
+                   const sr_reorder_params& p, cudaStream_t s, HostVec<uint64_t>& pairs_by_j,
+                   HostVec<uint32_t>& inter_h, HostVec<uint32_t>& uni_h, int64_t* E_out,
+                   HostVec<uint64_t>* pairs_by_key) {
   const bool dbg = getenv("SR_DEBUG_LSH") != nullptr;  // per-phase wall times (syncs the stream)
   double tl = 0;
   auto lap = [&](const char* what) {
@@ -441,7 +482,7 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
   sorted.release();
   if (pairs_by_key && E > (int64_t(1) << 26)) {  // the clustering's membership index above 2^26 pairs (R9)
     pairs_by_key->resize((size_t)E);
-    SR_CUDA_TRY(cudaMemcpyAsync(pairs_by_key->data(), allpairs.p, E * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    SR_TRY(d2h_staged(pairs_by_key->data(), allpairs.p, E * sizeof(uint64_t), s));
   }
   // exact Jaccard + heap-order sort
   DevBuf<uint32_t> d_inter(s), d_uni(s), idx_in(s), idx_out(s), i2(s), u2(s);
@@ -480,10 +521,9 @@ int lsh_candidates(const int64_t* rowptr_h, const int32_t* col_h, int64_t M, int
   pairs_by_j.resize((size_t)E);
   inter_h.resize((size_t)E);
   uni_h.resize((size_t)E);
-  SR_CUDA_TRY(cudaMemcpyAsync(pairs_by_j.data(), p2.p, E * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
-  SR_CUDA_TRY(cudaMemcpyAsync(inter_h.data(), i2.p, E * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-  SR_CUDA_TRY(cudaMemcpyAsync(uni_h.data(), u2.p, E * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-  SR_CUDA_TRY(cudaStreamSynchronize(s));
+  SR_TRY(d2h_staged(pairs_by_j.data(), p2.p, E * sizeof(uint64_t), s));
+  SR_TRY(d2h_staged(inter_h.data(), i2.p, E * sizeof(uint32_t), s));
+  SR_TRY(d2h_staged(uni_h.data(), u2.p, E * sizeof(uint32_t), s));
   lap("D2H");
   *E_out = E;
   return SR_OK;
