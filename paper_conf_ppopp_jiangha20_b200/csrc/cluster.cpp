@@ -519,6 +519,10 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
   if (spec && nthr >= 3 && init_pos > 0 && getenv("SR_CLUSTER_NOPIPE") == nullptr) {
     const int64_t nblocks = (int64_t)((init_pos + BS - 1) / BS);
     std::vector<Pre> ring[2] = {std::vector<Pre>(BS), std::vector<Pre>(BS)};
+    constexpr size_t kNodeAhead = 24;
+    // per 64 pops of a block: bit t set unless pop t was classified 1 (equal or deleted roots: a
+    // permanent skip), so the replay jumps over those pops without reading their records
+    std::vector<uint64_t> live[2] = {std::vector<uint64_t>(BS / 64 + 1), std::vector<uint64_t>(BS / 64 + 1)};
     SmallSet kset[2];  // keys re-inserted while replaying the previous / the current block
     int kprev = 0, kcur = 1;
     uint64_t fbits[2][1024];
@@ -553,6 +557,7 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
     const uint64_t* flush_keys = nullptr;
     int64_t flush_n = 0, eval_b0 = 0, eval_len = 0;
     Pre* eval_out = nullptr;
+    uint64_t* live_out = nullptr;
     // spin (the phase lasts about a second; yielding measured slower, r02l)
     auto pause = [] { __builtin_ia32_pause(); };
     std::atomic<int> team{0};
@@ -602,7 +607,7 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
         reinsert_pipe(c, key);
       }
     };
-    auto evaluate_one = [&](int64_t k, Pre& p) {
+    auto evaluate_one = [&](int64_t k, Pre& p) {  // (declared before its use in evaluate_chunk)
       const int32_t i = (int32_t)init[k].i, j = (int32_t)init[k].j;
       const int32_t pi = __atomic_load_n(&nd[i].parent, __ATOMIC_RELAXED);
       const int32_t pj = __atomic_load_n(&nd[j].parent, __ATOMIC_RELAXED);
@@ -632,6 +637,15 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
       p.uni = c.uni;
       p.cls = 3;
     };
+    // pops [k, e) of the current evaluation request, k a multiple of 64 (one live word)
+    auto evaluate_chunk = [&](int64_t k, int64_t e) {
+      uint64_t m = 0;
+      for (int64_t t = k; t < e; ++t) {
+        evaluate_one(eval_b0 + t, eval_out[t]);
+        if (eval_out[t].cls != 1) m |= 1ull << (t - k);
+      }
+      live_out[k >> 6] = m;
+    };
     // publish the next evaluation (the evaluators are idle: the previous one has completed)
     auto request = [&](int64_t b, const std::vector<uint64_t>* keys) {
       flush_n = keys ? (int64_t)keys->size() : 0;
@@ -641,6 +655,7 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
       eval_b0 = b * (int64_t)BS;
       eval_len = std::min<int64_t>((int64_t)init_pos, eval_b0 + (int64_t)BS) - eval_b0;
       eval_out = ring[b & 1].data();
+      live_out = live[b & 1].data();
       flush_done.store(0, std::memory_order_relaxed);
       eval_done.store(0, std::memory_order_relaxed);
       flush_cur.store((uint64_t)b << kTag, std::memory_order_release);
@@ -651,7 +666,7 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
       const double te = dbg ? now() : 0.0;
       if (team.load(std::memory_order_relaxed) < 2) {  // the runtime gave no evaluator thread
         for (int64_t t = 0; t < flush_n; ++t) members.insert_distinct_concurrent(flush_keys[t]);
-        for (int64_t t = 0; t < eval_len; ++t) evaluate_one(eval_b0 + t, eval_out[t]);
+        for (int64_t t = 0; t < eval_len; t += 64) evaluate_chunk(t, std::min<int64_t>(eval_len, t + 64));
         ready.store(b, std::memory_order_release);
       }
       while (ready.load(std::memory_order_acquire) != b) pause();
@@ -678,7 +693,7 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
             pause();
           while (claim(eval_cur, r, eval_len, 64, &k)) {
             const int64_t e = std::min(eval_len, k + 64);
-            for (int64_t t = k; t < e; ++t) evaluate_one(eval_b0 + t, eval_out[t]);
+            evaluate_chunk(k, e);
             if (eval_done.fetch_add(e - k, std::memory_order_acq_rel) + (e - k) == eval_len)
               ready.store(r, std::memory_order_release);
           }
@@ -697,8 +712,26 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
           overflow = false;
           if (b + 1 < nblocks) request(b + 1, b > 0 ? &kset[kprev].keys() : nullptr);
           const Pre* pr = ring[b & 1].data();
+          const uint64_t* lv = live[b & 1].data();
           const size_t b0 = (size_t)b * BS, b1 = std::min(init_pos, b0 + BS);
           for (size_t c = b0; c < b1 && nclusters > 0;) {
+            {  // jump over permanently skipped pops (class 1): no effect, whatever pops between
+              const size_t t = c - b0;
+              const uint64_t m = lv[t >> 6] >> (t & 63);
+              if (m == 0) {
+                const size_t nxt = b0 + ((t >> 6) + 1) * 64;
+                n_spec_used += (int64_t)(std::min(nxt, b1) - c);
+                c = nxt;
+                continue;
+              }
+              const size_t z = (size_t)__builtin_ctzll(m);
+              n_spec_used += (int64_t)z;
+              c += z;
+              if (c + kNodeAhead < b1) {  // the union-find nodes a pop a little ahead reads first
+                __builtin_prefetch(&nd[init[c + kNodeAhead].i]);
+                __builtin_prefetch(&nd[init[c + kNodeAhead].j]);
+              }
+            }
             if (!extra.empty() && !before(init[c], extra.top())) {  // a re-inserted pair pops first
               const int32_t i = (int32_t)extra.top().i, j = (int32_t)extra.top().j;
               extra.pop();
