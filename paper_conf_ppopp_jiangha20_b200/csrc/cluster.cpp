@@ -864,6 +864,14 @@ void cluster_rows(int64_t M, const int64_t* rowptr, const int32_t* col, int64_t 
         extra.pop();
       } else {
         if (zc < zero_keys.size() && (zero_new.empty() || zero_keys[zc] < zero_new.top())) {
+          if (zc + PF < zero_keys.size()) {  // the nodes (and their likely roots) of pops ahead
+            __builtin_prefetch(&nd[(int32_t)(zero_keys[zc + PF] >> 32)]);
+            __builtin_prefetch(&nd[(int32_t)(zero_keys[zc + PF] & 0xFFFFFFFFu)]);
+          }
+          if (zc + PF2 < zero_keys.size()) {
+            __builtin_prefetch(&nd[nd[(int32_t)(zero_keys[zc + PF2] >> 32)].parent]);
+            __builtin_prefetch(&nd[nd[(int32_t)(zero_keys[zc + PF2] & 0xFFFFFFFFu)].parent]);
+          }
           key = zero_keys[zc++];
         } else if (!zero_new.empty()) {
           key = zero_new.top();
