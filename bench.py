@@ -48,6 +48,14 @@ PAPER_CONTEXT = ("P100 (paper, P:334, P:350): ASpT-RR up to 2.91x SpMM vs best o
                  "up to 3.19x SDDMM vs ASpT-NR; geomean 1.19x / 1.49x (K=1024)")
 
 
+# ASpT panel height and dense-column threshold per workload (R17).  On C2, C3 and C5
+# the staged tiles lose to the L2 gather path at every threshold, so dense_min 64 keeps only
+# columns the whole 64-row panel shares (equal to no tiles); on the GNN matrix C4, 32-row panels
+# with columns shared by >= 4 rows beat the untiled plan by 7-8 % (profiles/r02/NOTES.md, r02aa).
+PLAN_DEFAULTS = {"gnn": dict(panel_rows=32, dense_min=4)}
+PLAN_DEFAULT = dict(panel_rows=64, dense_min=64)
+
+
 def parse(argv=None):
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -60,14 +68,15 @@ def parse(argv=None):
                     help="comma list of further K timed on the same plan (default: 32 for rmat at K=128; 'none')")
     ap.add_argument("--ops", default="spmm,sddmm")
     ap.add_argument("--mode", default="auto", choices=["auto", "force", "off"])
-    ap.add_argument("--panel-rows", type=int, default=64)
+    # plan parameters per workload (None = the config's default, PLAN_DEFAULTS below)
+    ap.add_argument("--panel-rows", type=int, default=None)
     ap.add_argument("--tile-cols", type=int, default=64)
     ap.add_argument("--max-bucket", type=int, default=32)
     # ASpT dense-column threshold (R17).  The paper's example is 2 (a P100 with 64 KB of
     # shared memory per SM); on B200 (126 MB L2, row-group task kernels gathering from L2 at ~15 TB/s)
     # staging pays only for columns shared by (nearly) the whole 64-row panel: sweeps in
     # profiles/r01/NOTES.md (session 3: 64 best with tiles present, equal to no tiles).
-    ap.add_argument("--dense-min", type=int, default=64)
+    ap.add_argument("--dense-min", type=int, default=None)
     # dense criterion of the AUTO round-1 decision (R28): a column shared by 1/8 of the panel
     ap.add_argument("--auto-dense-min", type=int, default=8)
     ap.add_argument("--e2e-steps", type=int, default=3)
@@ -81,7 +90,11 @@ def parse(argv=None):
     ap.add_argument("--plan-cache", default=None,
                     help="experiments only: load the plan image from this file if present, else save it there "
                          "(preprocess then reports the load, not the reorder)")
-    return ap.parse_args(argv)
+    args = ap.parse_args(argv)
+    for k, v in PLAN_DEFAULTS.get(args.config, PLAN_DEFAULT).items():
+        if getattr(args, k) is None:
+            setattr(args, k, v)
+    return args
 
 
 def measured_peaks():

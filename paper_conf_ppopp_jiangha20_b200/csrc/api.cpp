@@ -510,19 +510,14 @@ int build_exec_plan_into(sr_csr_s* h, int64_t pb, int64_t pe, cudaStream_t s, De
   P.dscratch.release();
   P.dscratch_k = 0;
   // persistent phase-D CTAs take units round-robin: largest first balances them; every unit
-  // gets a producer blob (DUnit | VTiles | dense column ids), 16-byte aligned
+  // gets a producer blob (DUnit | VTiles), 16-byte aligned
   std::stable_sort(units.begin(), units.end(), [](const DUnit& a, const DUnit& b) { return a.nvt > b.nvt; });
   std::vector<int4> blobs;
   std::vector<int2> blob_meta;
   for (const DUnit& u : units) {
-    const VTile& v0 = vtiles[u.vt0];
-    const VTile& vl = vtiles[u.vt0 + u.nvt - 1];
-    const int32_t col_lo = v0.col0, ncol = vl.col0 + vl.ncols - col_lo;
-    std::vector<int32_t> rec(8 + 4 * u.nvt + ncol, 0);
+    std::vector<int32_t> rec(8 + 4 * u.nvt, 0);
     std::memcpy(rec.data(), &u, sizeof(DUnit));
     std::memcpy(rec.data() + 8, &vtiles[u.vt0], sizeof(VTile) * u.nvt);
-    std::copy(T.dense_cols.begin() + col_lo, T.dense_cols.begin() + col_lo + ncol, rec.begin() + 8 + 4 * u.nvt);
-    while (rec.size() % 4) rec.push_back(0);
     blob_meta.push_back(make_int2((int)blobs.size(), (int)(rec.size() * 4)));
     for (size_t w = 0; w < rec.size(); w += 4) blobs.push_back(make_int4(rec[w], rec[w + 1], rec[w + 2], rec[w + 3]));
   }

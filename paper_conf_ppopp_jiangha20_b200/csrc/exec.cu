@@ -821,7 +821,7 @@ constexpr int kSpmmStages = SR_SPMM_STAGES;
 constexpr int kSddmmStages = 2;               // SDDMM stages also carry output indices
 constexpr int kMaxStages = kSpmmStages > kSddmmStages ? kSpmmStages : kSddmmStages;
 constexpr int kDenseCtasPerSM = SR_DENSE_CTAS;
-constexpr size_t kUnitBlobBytes = kMaxUnitBlobBytes;  // DUnit + VTiles + dense column ids
+constexpr size_t kUnitBlobBytes = kMaxUnitBlobBytes;  // DUnit + VTiles
 
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
@@ -855,6 +855,9 @@ struct StageLayout {
   __host__ size_t smem(int nst_) const { return 128 + (size_t)nst_ * bytes() + 2 * kUnitBlobBytes; }
 };
 
+static_assert(kMaxExecTile <= 128, "the producer's lanes stage four tile columns each");
+static_assert(kMaxUnitTiles <= 32, "the producer holds one VTile of its unit per lane");
+
 // Producer warp: every tile of every unit of this CTA.
 __device__ __forceinline__ void dense_produce(const DUnit* __restrict__ units, int n_units,
                                               const VTile* __restrict__ vtiles,
@@ -869,9 +872,10 @@ __device__ __forceinline__ void dense_produce(const DUnit* __restrict__ units, i
   const size_t SB = L.bytes();
   const int npass = (K + KCP - 1) / KCP;
   // This CTA's units are blockIdx.x + k·gridDim.x (units are sorted by decreasing size, so the
-  // round robin balances).  Everything the producer needs about a unit — its DUnit, its
-  // VTiles and its dense column ids — is one contiguous 16-byte-aligned blob, fetched by one
-  // bulk copy two units ahead into a 2-slot ring: no dependent global load on the issue path.
+  // round robin balances).  A unit's DUnit and VTiles (<= 32, one per lane) are one contiguous
+  // 16-byte-aligned blob, fetched by one bulk copy two units ahead into a 2-slot ring; a tile's
+  // dense column ids are loaded from global memory before the producer waits for the tile's
+  // stage to drain, so their latency hides behind the consumers.
   char* ring = smem + L.nst * SB;
   const int nmine = ((int)blockIdx.x < n_units) ? (n_units - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x : 0;
   auto fetch_blob = [&](int k, int2 m) {
@@ -891,18 +895,23 @@ __device__ __forceinline__ void dense_produce(const DUnit* __restrict__ units, i
     const DUnit u = *reinterpret_cast<const DUnit*>(blob);
     const bool last_unit = k == nmine - 1;
     const VTile mine = lane < u.nvt ? reinterpret_cast<const VTile*>(blob + sizeof(DUnit))[lane] : VTile{0, 0, 0, 0};
-    const int col_lo = __shfl_sync(FULL, mine.col0, 0);
-    const int32_t* ucols = reinterpret_cast<const int32_t*>(blob + sizeof(DUnit) + u.nvt * sizeof(VTile));
     for (int pass = 0; pass < npass; ++pass) {
       const int k0 = pass * KCP, kw = min(KCP, K - k0);
       for (int ti = 0; ti < u.nvt; ++ti, ++idx) {
         const int st = idx % L.nst;
-        if (idx >= L.nst) mbar_wait(&empty[st], ((idx - L.nst) / L.nst) & 1);
         VTile v;
         v.ent0 = __shfl_sync(FULL, mine.ent0, ti);
         v.nent = __shfl_sync(FULL, mine.nent, ti);
         v.col0 = __shfl_sync(FULL, mine.col0, ti);
         v.ncols = __shfl_sync(FULL, mine.ncols, ti);
+        // this lane's four column ids (tile columns 4·lane .. 4·lane+3; a ragged group repeats
+        // its first row), in flight while the stage drains
+        int cid[4] = {0, 0, 0, 0};
+        if (lane * 4 < v.ncols) {
+#pragma unroll
+          for (int q = 0; q < 4; ++q) cid[q] = __ldg(dense_cols + v.col0 + min(lane * 4 + q, v.ncols - 1));
+        }
+        if (idx >= L.nst) mbar_wait(&empty[st], ((idx - L.nst) / L.nst) & 1);
         char* base = smem + st * SB;
         if (lane == 0) {
           StageHdr* h = reinterpret_cast<StageHdr*>(base + L.hdr_off());
@@ -920,7 +929,7 @@ __device__ __forceinline__ void dense_produce(const DUnit* __restrict__ units, i
         }
         if (!L.bulk) {  // unaligned operands (scalar path): plain loads and shared stores
           float* bs = reinterpret_cast<float*>(base + L.b_off());
-          const int32_t* cols = ucols + (v.col0 - col_lo);
+          const int32_t* cols = dense_cols + v.col0;
           for (int i = lane; i < v.ncols * kw; i += 32) {
             const int j = i / kw, k = i - j * kw;
             bs[(size_t)j * KCP + k] = __ldg(src + (int64_t)cols[j] * ld + k0 + k);
@@ -941,22 +950,20 @@ __device__ __forceinline__ void dense_produce(const DUnit* __restrict__ units, i
         const uint32_t bytes = row_bytes + (uint32_t)(L.trp_ints * 4 + v.nent * 8 + (L.oidx ? v.nent * 4 : 0));
         if (lane == 0) mbar_expect_tx(&full[st], bytes);
         __syncwarp();
-        const int32_t* cols = ucols + (v.col0 - col_lo);
         if (tmap) {
           // TMA gather4: one instruction stages four dense-column rows (box = KCP columns × 1 row
-          // of the row-major operand, 4 row coordinates); a ragged last group repeats a row
-          for (int j4 = lane; j4 * 4 < v.ncols; j4 += 32) {
-            const int j = j4 * 4;
-            const int c0 = cols[j];
-            const int c1 = j + 1 < v.ncols ? cols[j + 1] : c0;
-            const int c2 = j + 2 < v.ncols ? cols[j + 2] : c0;
-            const int c3 = j + 3 < v.ncols ? cols[j + 3] : c0;
-            tma_gather4(base + L.b_off() + (size_t)j * KCP * 4, tmap, k0, c0, c1, c2, c3, &full[st]);
+          // of the row-major operand, 4 row coordinates); tiles have <= 64 columns = 16 lanes
+          if (lane * 4 < v.ncols)
+            tma_gather4(base + L.b_off() + (size_t)lane * 4 * KCP * 4, tmap, k0, cid[0], cid[1], cid[2], cid[3],
+                        &full[st]);
+        } else {  // one bulk copy per row: lane l stages rows 4l .. 4l+3
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            const int j = lane * 4 + q;
+            if (j < v.ncols)
+              bulk_g2s(base + L.b_off() + (size_t)j * KCP * 4, src + (int64_t)cid[q] * ld + k0, (uint32_t)(kw * 4),
+                       &full[st]);
           }
-        } else {
-          for (int j = lane; j < v.ncols; j += 32)
-            bulk_g2s(base + L.b_off() + (size_t)j * KCP * 4, src + (int64_t)cols[j] * ld + k0, (uint32_t)(kw * 4),
-                     &full[st]);
         }
         if (lane == 0)
           bulk_g2s(base + L.trp_off(), trp + (int64_t)vt * L.trp_ints, (uint32_t)(L.trp_ints * 4), &full[st]);
@@ -1075,16 +1082,22 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) spmm_
     }
     if ((hd.flags & kLastOfUnit) && hd.split >= 0) {
       // giant panel split over several units: the last unit to finish sums the chunk
-      // partials in unit order (deterministic) and writes the panel's dense rows
-      __threadfence();
+      // partials in unit order (deterministic) and writes the panel's dense rows.  Release /
+      // acquire through one thread: the consumers' partial stores happen before thread 0's
+      // gpu-scope fence (CTA barrier), its ticket follows the fence; the last unit's thread 0
+      // fences after its ticket and the barrier orders every consumer's L2 reads (ld.cg) after
+      // (one fence per unit instead of one per consumer thread: each is a CCTL.IVALL of L1)
       consumers_sync();
       const int2 si = split_info[hd.split];
-      if (threadIdx.x == 0) last_ticket = (atomicAdd(split_counter + si.x, 1) == si.y - 1);
+      if (threadIdx.x == 0) {
+        __threadfence();
+        last_ticket = (atomicAdd(split_counter + si.x, 1) == si.y - 1);
+        if (last_ticket) __threadfence();
+      }
       consumers_sync();
       if (last_ticket) {
         // all consumer threads share the (row, fragment) sums; chunk partials are added
         // in chunk order with 4 loads in flight (a hub panel can have >100 chunks)
-        __threadfence();
         const int kq = (K + VEC - 1) / VEC;
         for (int item = threadIdx.x; item < hd.nrows * kq; item += kDenseWarps * 32) {
           const int r = item / kq, k = (item - r * kq) * VEC;

@@ -154,11 +154,12 @@ struct __align__(16) DUnit {
 constexpr int kRtMaxRows = 8;                        // register-tile engine: panel rows
 constexpr int64_t kRtChunk = 1024;                   // register-tile stream entries per warp (chunk)
 constexpr int32_t kRtHeader = (int32_t)0x80000000u;  // marks a column header entry
-constexpr int kMaxUnitTiles = 8;
+constexpr int kMaxUnitTiles = 32;  // one VTile per producer lane; whole panels of <= 2048 dense
+                                   // columns are one unit (no split partials / combine)
 constexpr int kMaxExecTile = 64;
 constexpr int kMaxTileEntries = 384;  // SpMM: 3 stages + blob ring must fit twice per SM
-// producer-side record of a unit: DUnit, its VTiles, its dense column ids (16-byte aligned)
-constexpr int kMaxUnitBlobBytes = 32 + kMaxUnitTiles * 16 + kMaxUnitTiles * kMaxExecTile * 4;
+// producer-side record of a unit: DUnit and its VTiles (16-byte aligned)
+constexpr int kMaxUnitBlobBytes = 32 + kMaxUnitTiles * 16;
 
 struct TmapKey {
   const void* base = nullptr;

@@ -206,6 +206,34 @@ def test_register_tiles_split_hub_panels(env, oracle, K):
     np.testing.assert_array_equal(C, C2)
 
 
+@pytest.mark.parametrize("K", [128, 256])
+def test_tma_engine_split_hub_panel(env, oracle, K):
+    """A 16-row panel with 5000 shared columns: 79 staged tiles of 64 columns, more than one
+    phase-D unit holds (32 tiles), so the panel runs as three units whose partial sums the
+    last one adds in unit order (release / acquire through one thread per CTA)."""
+    sr, _ = env
+    rng = np.random.default_rng(5)
+    n, m = 64, 9000
+    rows, cols = [], []
+    hub = rng.choice(m, size=5000, replace=False)
+    for i in range(n):
+        if i < 16:
+            rows.append(np.full(hub.size, i))
+            cols.append(hub)
+        d = int(rng.integers(0, 30))
+        extra = np.setdiff1d(rng.choice(m, size=d, replace=False), hub if i < 16 else [])
+        rows.append(np.full(extra.size, i))
+        cols.append(extra)
+    rowptr, colidx = g._from_coo(n, m, np.concatenate(rows), np.concatenate(cols))
+    A = g.CSR(n, m, rowptr, colidx, g._uniform_vals(colidx.size, 4))
+    M, B, X, Y, C, out = _run(env, A, K, sr.default_params(**dict(_plan_kw(16, 2, 0)), tile_cols=64))
+    assert M.stats()["dense1"] >= 16 * 5000
+    _spmm_check(oracle, A, B, C)
+    _sddmm_check(oracle, A, X, Y, out)
+    _, _, _, _, C2, _ = _run(env, A, K, sr.default_params(**dict(_plan_kw(16, 2, 0)), tile_cols=64))
+    np.testing.assert_array_equal(C, C2)  # deterministic ordered combine
+
+
 def test_unsorted_input_keeps_caller_nnz_order(env, oracle):
     sr, _ = env
     A = g.random_csr(120, 90, 0.1, 12, empty_frac=0.1)
@@ -388,10 +416,14 @@ def test_full_size_plan_bench_params(env, oracle, config):
     round 2 on C5); SpMM (K=128) on 2000 sampled rows + the 20 longest, SDDMM on all their nnz.
     C5's round 2 at max_bucket 32 has E2 = 275 M candidates, beyond what the oracle's plain
     priority queue clusters in minutes: C5 runs here with max_bucket 8, and its bench-parameter
-    plan is checked by test_full_size_cf_bench_params."""
+    plan is checked by test_full_size_cf_bench_params.  C4 runs bench.py's per-config plan
+    parameters (32-row panels, dense_min 4: half its nnz on the phase-D TMA engine)."""
     sr, torch = env
     A = g.make(config)
-    kw = dict(BENCH_KW, max_bucket=8) if config == "cf" else BENCH_KW
+    import bench
+    kw = dict(BENCH_KW, **bench.PLAN_DEFAULTS.get(config, {}))  # C4: 32-row panels, dense_min 4
+    if config == "cf":
+        kw["max_bucket"] = 8
     M = sr.SparseMatrix.from_csr(A)
     M.reorder(sr.default_params(**kw))
     ref = oracle.plan(A, **kw)
