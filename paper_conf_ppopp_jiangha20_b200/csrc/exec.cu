@@ -813,12 +813,15 @@ __global__ void __launch_bounds__(256) sddmm_rtile_scalar_kernel(
 #ifndef SR_SPMM_STAGES
 #define SR_SPMM_STAGES 3
 #endif
+#ifndef SR_SDDMM_STAGES
+#define SR_SDDMM_STAGES 3
+#endif
 #ifndef SR_DENSE_CTAS
 #define SR_DENSE_CTAS 2
 #endif
 constexpr int kDenseWarps = SR_DENSE_WARPS;  // consumer warps per phase-D CTA (+1 producer warp)
 constexpr int kSpmmStages = SR_SPMM_STAGES;
-constexpr int kSddmmStages = 2;               // SDDMM stages also carry output indices
+constexpr int kSddmmStages = SR_SDDMM_STAGES;  // SDDMM stages also carry output indices (3 fit since r02aa)
 constexpr int kMaxStages = kSpmmStages > kSddmmStages ? kSpmmStages : kSddmmStages;
 constexpr int kDenseCtasPerSM = SR_DENSE_CTAS;
 constexpr size_t kUnitBlobBytes = kMaxUnitBlobBytes;  // DUnit + VTiles
@@ -1142,7 +1145,7 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) sddmm
     const int32_t* __restrict__ d_oidx, const int32_t* __restrict__ pos_xrow, const float* __restrict__ X,
     int64_t ldx, const float* __restrict__ Y, int64_t ldy, int K, int TW, int TS, float* __restrict__ out,
     const int4* __restrict__ blobs, const int2* __restrict__ blob_meta, const __grid_constant__ CUtensorMap tmap,
-    int use_tmap, int dbg) {
+    int use_tmap, int dbg, int nst) {
   constexpr int G = 32 / LPG;
   constexpr int KC = LPG * VEC;   // columns of one chunk
   constexpr int KCP = NCH * KC;   // columns staged per pass (slot stride)
@@ -1151,7 +1154,7 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) sddmm
   __shared__ uint64_t full[kMaxStages + 2], empty[kMaxStages];
   const int lane = threadIdx.x & 31, g = lane / LPG, lg = lane % LPG;
   const int warp = threadIdx.x >> 5;
-  const StageLayout L{((TW + 3) & ~3) * KCP, TS, true, kSddmmStages, dbg >> 1, (dbg & 1) != 0};
+  const StageLayout L{((TW + 3) & ~3) * KCP, TS, true, nst, dbg >> 1, (dbg & 1) != 0};
   dense_init_barriers(full, empty);
   if (warp == kDenseWarps) {
     dense_produce(units, n_units, vtiles, dense_cols, trp, ent, d_oidx, Y, ldy, K, KCP, L, smem, full, empty,
@@ -1192,23 +1195,31 @@ __global__ void __launch_bounds__((kDenseWarps + 1) * 32, kDenseCtasPerSM) sddmm
             const int j = bse + uu * G + g;
             en[uu] = j < b1 ? es[j] : make_int2(0, 0);
           }
+          // only groups that hold an entry read a staged row, and steps past the row's last
+          // entry are skipped (warp-uniform): a row has ~4-5 entries of a tile on C5 against the
+          // G·U = 16 slots of a batch, and every idle slot used to read slot 0 of the stage —
+          // 10 shared-memory wavefronts per nnz, the SM's shared-memory pipe 90 % busy (r02af)
 #pragma unroll
           for (int uu = 0; uu < U; ++uu) {
             float d = 0.f;
+            if (bse + uu * G + g < b1) {
 #pragma unroll
-            for (int c = 0; c < NCH; ++c) {
-              if (c * KC + lg * VEC < kw) {
-                Frag<VEC> y;
-                y.load_s(tile + (size_t)en[uu].x * KCP + c * KC + lg * VEC);
-                d += x[c].dot(y);
+              for (int c = 0; c < NCH; ++c) {
+                if (c * KC + lg * VEC < kw) {
+                  Frag<VEC> y;
+                  y.load_s(tile + (size_t)en[uu].x * KCP + c * KC + lg * VEC);
+                  d += x[c].dot(y);
+                }
               }
             }
             part[uu] = d;
           }
 #pragma unroll
           for (int uu = 0; uu < U; ++uu) {
+            if (bse + uu * G < b1) {
 #pragma unroll
-            for (int off = LPG / 2; off > 0; off >>= 1) part[uu] += __shfl_xor_sync(FULL, part[uu], off);
+              for (int off = LPG / 2; off > 0; off >>= 1) part[uu] += __shfl_xor_sync(FULL, part[uu], off);
+            }
           }
           if (lg == 0) {
 #pragma unroll
@@ -1489,8 +1500,12 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
   }
   if (P.n_units > 0) {
     const int TW = P.tile_cols;
-    const size_t smem =
-        StageLayout{((TW + 3) & ~3) * NCH_D * KC, P.trp_stride, true, kSddmmStages, 0, true}.smem(kSddmmStages);
+    // ring depth: kSddmmStages (3 since the unit blobs shrank, r02ad: −9-11 % per dense nnz on C5)
+    // while two CTAs fit an SM, else 2
+    const StageLayout SL{((TW + 3) & ~3) * NCH_D * KC, P.trp_stride, true, kSddmmStages, 0, true};
+    int nst = kSddmmStages;
+    while (nst > 2 && (size_t)kDenseCtasPerSM * (SL.smem(nst) + 1024) > 233472) --nst;
+    const size_t smem = SL.smem(nst);
     CUtensorMap tmap;
     const int use_tmap = (VEC == 4 && cached_row_gather_map(P, &tmap, Y, h->A.N, K, ldy, NCH_D * KC)) ? 1 : 0;
     const unsigned grid = (unsigned)std::min<int64_t>(P.n_units, (int64_t)kDenseCtasPerSM * num_sms());
@@ -1499,11 +1514,16 @@ int run_sddmm(sr_csr_s* h, const float* X, int64_t ldx, const float* Y, int64_t 
       SR_TRY(raise_smem_limit(reinterpret_cast<const void*>(kern), smem));
       kern<<<grid, (kDenseWarps + 1) * 32, smem, s>>>(
           P.units.p, (int)P.n_units, P.vtiles.p, P.dense_cols.p, P.trp.p, P.d_ent.p, P.d_oidx.p, P.pos_xrow.p, X, ldx,
-          Y, ldy, (int)K, TW, P.trp_stride, out, P.blobs.p, P.blob_meta.p, tmap, use_tmap, flags);
+          Y, ldy, (int)K, TW, P.trp_stride, out, P.blobs.p, P.blob_meta.p, tmap, use_tmap, flags, nst);
       SR_CUDA_TRY(cudaGetLastError());
       return SR_OK;
     };
-    constexpr int UD = 4;
+    // entry slots per group and batch of the SDDMM phase-D consumer (measurement knob; 1 measured
+    // best: a row holds ~4-5 entries of a tile, C5 dense 1.47 / 1.41 / 1.29 ms at U 4 / 2 / 1, r02ah)
+#ifndef SR_SDDMM_DENSE_U
+#define SR_SDDMM_DENSE_U 1
+#endif
+    constexpr int UD = SR_SDDMM_DENSE_U;
     if (P.profiling) SR_TRY(prof_begin(P, 3, s));
     const int rpw = dense_rows_per_warp(P.panel_rows);
     if (rpw <= 2) SR_TRY(launch(sddmm_dense_kernel<LPG, VEC, UD, NCH_D, 2>));
