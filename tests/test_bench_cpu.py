@@ -40,6 +40,17 @@ def test_gpus_flag_fails_loudly_without_enough_gpus():
     assert "--gpus 2" in r.stderr and "device" in r.stderr
 
 
+def test_plan_parameters_per_config():
+    """The GNN matrix runs its measured tiled plan (32-row panels, dense_min 4: phase D beats the
+    untiled plan there, profiles/r02/NOTES.md r02aa); the others keep dense_min 64; explicit flags win."""
+    a = bench.parse(["--config", "gnn"])
+    assert (a.panel_rows, a.dense_min) == (32, 4)
+    a = bench.parse([])
+    assert (a.config, a.panel_rows, a.dense_min) == ("rmat", 64, 64)
+    a = bench.parse(["--config", "gnn", "--panel-rows", "16", "--dense-min", "3"])
+    assert (a.panel_rows, a.dense_min) == (16, 3)
+
+
 def test_sddmm_bytes_count_output_write():
     tm = dict(sparse_nnz=10, sparse_items=2, sparse_distinct_cols=3, sparse_rows=2, zero_rows=1, rmw_rows=0,
               dense_nnz=4, dense_distinct_cols=1, dense_rows=1, sparse_group_loads=5, dense_col_loads=1)
